@@ -1,0 +1,348 @@
+#!/usr/bin/env python
+"""Benchmark of the PLR hot path on B200 (contract in the task statement).
+
+Workload (BASELINE.json configs[1]): the 2- and 3-tuple int32 prefix sums
+(1: 0, 1) and (1: 0, 0, 1) on n = 2^30 seeded random int32 per GPU.  One
+step = one pass of the whole hot path (plan already built: fused load/FIR,
+per-thread chunks, warp/block propagation, decoupled look-back, correction,
+store) for each of the two signatures over the resident input.  Metric:
+effective GB/s = (bytes read + bytes written) / time = 8 B/element, as in
+BASELINE.json ("effective GB/s (read+write) and elements/s").  Inputs are
+4 GiB per tensor, far larger than the 126 MB L2, so no flush is needed.
+
+N > 1 (torchrun): each rank holds a 2^30-element contiguous segment of one
+long sequence (weak scaling); a step is the sharded evaluation
+(plr_execute_sharded: local pass, one 64-byte NCCL allgather, fixup/seeded
+pass); the time is the max over ranks.
+
+--impl reference: the CPU oracle (oracle/, the plain sequential Eq. (1)) timed
+as it stands on this host's cores on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads  # noqa: E402
+
+WORKLOAD_SIGS = ("tuple2", "tuple3")
+N_FULL = 1 << 30
+METRIC = "effective GB/s (read+write) and elements/s vs memcpy/HBM peak at 1/2/4/8 B200"
+BYTES_PER_ELT = 8
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="plr", choices=["plr", "reference"])
+    ap.add_argument("--n", type=int, default=N_FULL)
+    ap.add_argument("--no-extras", action="store_true", help="skip per-signature table / e2e / cpu baseline")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0}, "fallback"
+
+
+def ncu_traffic():
+    """dram bytes per launch of the scan kernel from the committed ncu summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_scan_traffic.json")
+    try:
+        with open(p) as f:
+            return json.load(f)
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------ clocks --
+class ClockSampler:
+    """NVML sampling of SM clock and throttle reasons during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, index):
+        self.samples = []
+        self.reasons = 0
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        rs = [name for bit, name in self.REASONS.items() if self.reasons & bit and name != "gpu_idle"]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": rs, "samples": len(self.samples)}
+
+
+# --------------------------------------------------------------- reference --
+def run_reference(args, rank, world):
+    import numpy as np
+    import oracle
+    if rank != 0:
+        return
+    sample = 1 << 24                      # per signature per step, bounded
+    xs = {}
+    for name in WORKLOAD_SIGS:
+        sig = workloads.BY_NAME[name]
+        xs[name] = workloads.host_input(sample, sig.dtype, workloads.seed_for(1))
+    for _ in range(args.warmup):
+        for name in WORKLOAD_SIGS:
+            sig = workloads.BY_NAME[name]
+            oracle.recurrence(xs[name], sig.a, sig.b, sig.dtype)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        for name in WORKLOAD_SIGS:
+            sig = workloads.BY_NAME[name]
+            oracle.recurrence(xs[name], sig.a, sig.b, sig.dtype)
+    dt = time.perf_counter() - t0
+    elems = args.steps * sample * len(WORKLOAD_SIGS)
+    gbs = elems * BYTES_PER_ELT / dt / 1e9
+    desc = "first 2^24 elements of the workload input per signature per step, sequential C oracle (gcc -O2), 1 thread"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+        "data": "synthetic (seeded uniform int32)",
+        "config": {"workload": "configs[1] tuple prefix sums (1:0,1)+(1:0,0,1), bounded sample", "n_per_sig": sample},
+        "elements_per_s": elems / dt,
+        "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc},
+        "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# -------------------------------------------------------------------- main --
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", args.gpus))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import numpy as np
+    import torch
+    import paper_conf_asplos_malekib18_b200 as plr
+
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n = args.n
+    peaks, peaks_src = measured_peaks()
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+
+    plans = {name: plr.Plan(workloads.BY_NAME[name].a, workloads.BY_NAME[name].b, "int32", n_max=n)
+             for name in WORKLOAD_SIGS}
+    x = workloads.device_input(n, "int32", workloads.seed_for(1, rank))
+    y = torch.empty_like(x)
+    stream = torch.cuda.current_stream()
+    comm = plr.ShardComm() if world > 1 else None
+
+    def step(kernel_events=None):
+        for name in WORKLOAD_SIGS:
+            if kernel_events is not None:
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+            if comm is None:
+                plans[name](x, y)
+            else:
+                plans[name].sharded(x, y, comm=comm)
+            if kernel_events is not None:
+                e1.record(stream)
+                kernel_events.append((e0, e1))
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(torch.cuda.current_device())
+    start = torch.cuda.Event(enable_timing=True)
+    end = torch.cuda.Event(enable_timing=True)
+    kev = []
+    with sampler:
+        start.record(stream)
+        for _ in range(args.steps):
+            step(kev)
+        end.record(stream)
+        torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    ms = start.elapsed_time(end)
+    if dist:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    ms_step = ms / args.steps
+    elems_step = n * len(WORKLOAD_SIGS) * world
+    gbs = elems_step * BYTES_PER_ELT / (ms_step * 1e-3) / 1e9
+    kern_ms = [a.elapsed_time(b) for a, b in kev]
+    kern_avg = sum(kern_ms) / len(kern_ms)
+
+    extras = {}
+    if rank == 0 and world == 1 and not args.no_extras:
+        extras = run_extras(args, plr, torch, np, n, x, y, plans, hbm)
+    if rank == 0:
+        traffic = ncu_traffic()
+        achieved = n * BYTES_PER_ELT / (kern_avg * 1e-3) / 1e9
+        line = {
+            "metric": METRIC, "value": round(gbs, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": max(3, args.warmup), "ms_per_step": round(ms_step, 4), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic (seeded uniform int32)",
+            "config": {"workload": "BASELINE configs[1]: (1: 0, 1) and (1: 0, 0, 1) int32 tuple prefix sums, "
+                                   "n=2^30 per GPU, one launch per signature per step",
+                       "n_per_gpu": n, "signatures": [workloads.BY_NAME[s].text() for s in WORKLOAD_SIGS],
+                       "l2": "inputs 4 GiB per tensor >> 126 MB L2 (no flush needed)",
+                       "tile_elems": plans[WORKLOAD_SIGS[0]].info["tile_elems"],
+                       "ctas_per_sm": plans[WORKLOAD_SIGS[0]].info["ctas_per_sm"]},
+            "elements_per_s": elems_step / (ms_step * 1e-3),
+            "frac_of_hbm_peak": round(gbs / world / hbm, 4),
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
+                         "frac": round(achieved / hbm, 4),
+                         "traffic": (traffic or {}).get("bytes_per_launch"),
+                         "peak_source": "MEASURED_PEAKS.json hbm_gbs (%s)" % peaks_src,
+                         "kernel": "plr_scan_kernel (single pass), avg of %d launches, CUDA events on the launch stream"
+                                   % len(kern_ms),
+                         "kernel_ms": round(kern_avg, 4),
+                         "algorithmic_bytes_per_launch": n * BYTES_PER_ELT},
+            "gpu_launches": args.steps * len(WORKLOAD_SIGS) * (1 if world == 1 else 6),
+            "clocks": sampler.summary(),
+        }
+        line.update(extras)
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.close()
+    if dist:
+        dist.destroy_process_group()
+
+
+def run_extras(args, plr, torch, np, n, x, y, plans, hbm):
+    """Per-signature table, in-run memcpy yardstick, e2e through host memory,
+    and the CPU oracle baseline."""
+    out = {}
+    stream = torch.cuda.current_stream()
+
+    def time_it(fn, reps=10, warm=3):
+        for _ in range(warm):
+            fn()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(reps):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / reps
+
+    # memcpy yardstick: device-to-device copy of the same 4n bytes
+    ms_cp = time_it(lambda: y.copy_(x))
+    memcpy_gbs = n * BYTES_PER_ELT / (ms_cp * 1e-3) / 1e9
+    out["memcpy_gbs"] = round(memcpy_gbs, 1)
+
+    # every Table-1 signature at the bench size
+    table = {}
+    xf = workloads.device_input(n, "float32", workloads.seed_for(4))
+    for sig in workloads.TABLE1:
+        plan = plans.get(sig.name) or plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+        xin = x if sig.dtype == "int32" else xf
+        yout = y if sig.dtype == "int32" else torch.empty_like(xf)
+        ms = time_it(lambda: plan(xin, yout))
+        g = n * BYTES_PER_ELT / (ms * 1e-3) / 1e9
+        table[sig.name] = {"sig": sig.text(), "ms": round(ms, 4), "GB/s": round(g, 1),
+                           "Gelem/s": round(n / (ms * 1e-3) / 1e9, 1),
+                           "frac_memcpy": round(g / memcpy_gbs, 4), "frac_hbm_peak": round(g / hbm, 4)}
+        if sig.name not in plans:
+            plan.close()
+        del yout
+    del xf
+    torch.cuda.empty_cache()
+    out["per_signature"] = table
+
+    # e2e: through the C ABI with pinned HOST buffers; H2D + D2H inside the timing
+    xh = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    xh.copy_(x)
+    yh = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    def e2e_step():
+        for name in WORKLOAD_SIGS:
+            plans[name].execute_host(xh, yh)
+    e2e_step()
+    steps = max(1, min(args.steps, 5))
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        e2e_step()
+    dt = (time.perf_counter() - t0) / steps
+    out["e2e"] = {"value": round(n * len(WORKLOAD_SIGS) * BYTES_PER_ELT / dt / 1e9, 2), "unit": "GB/s",
+                  "h2d_bytes_per_step": n * 4 * len(WORKLOAD_SIGS), "d2h_bytes_per_step": n * 4 * len(WORKLOAD_SIGS),
+                  "ms_per_step": round(dt * 1e3, 2), "steps": steps,
+                  "path": "plr_execute_host: pinned host -> 32 Mi-element chunks, H2D/compute/D2H overlapped"}
+
+    # CPU oracle baseline on a bounded sample of the same input
+    import oracle
+    sample = 1 << 28
+    xs = x[:sample].cpu().numpy()
+    t0 = time.perf_counter()
+    for name in WORKLOAD_SIGS:
+        sig = workloads.BY_NAME[name]
+        oracle.recurrence(xs, sig.a, sig.b, sig.dtype)
+    dt = time.perf_counter() - t0
+    cg = sample * len(WORKLOAD_SIGS) * BYTES_PER_ELT / dt / 1e9
+    out["cpu_baseline"] = {"value": round(cg, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                           "sample": "first 2^28 elements of the workload input, each of the 2 signatures, "
+                                     "sequential C oracle (gcc -O2), 1 thread, %.1f s" % dt,
+                           "host_cores_available": os.cpu_count()}
+    return out
+
+
+if __name__ == "__main__":
+    main()

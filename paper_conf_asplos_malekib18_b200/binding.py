@@ -1,0 +1,264 @@
+"""ctypes binding of libplr_b200.so (include/plr.h).  Marshalling only."""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libplr_b200.so")
+PAYLOAD_BYTES = 64
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        "libplr_b200.so is not built (run `python -c 'import __graft_entry__ as g; g.build()'` or "
+        "`python paper_conf_asplos_malekib18_b200/build.py`); there is no fallback path")
+
+lib = ctypes.CDLL(LIB_PATH)
+
+_P = ctypes.c_void_p
+_S = ctypes.c_size_t
+_I = ctypes.c_int
+_st = ctypes.c_int
+
+_SIGS = {
+    "plr_plan_create": ([ctypes.POINTER(_P), _P, _I, _P, _I, _I, _S], _st),
+    "plr_plan_destroy": ([_P], _st),
+    "plr_plan_get_info": ([_P, _P], _st),
+    "plr_plan_factor_lists": ([_P, ctypes.c_int64, _P], _st),
+    "plr_execute": ([_P, _P, _P, _S, _P], _st),
+    "plr_execute_continue": ([_P, _P, _P, _S, _P, _P, _P], _st),
+    "plr_reduce": ([_P, _P, _S, _P, _P], _st),
+    "plr_payload_from_output": ([_P, _P, _P, _S, _P, _P], _st),
+    "plr_combine": ([_P, _P, _I, _I, _P, _P], _st),
+    "plr_combine_host": ([_P, _P, _I, _I, _P], _st),
+    "plr_fixup": ([_P, _P, _S, _P, _P], _st),
+    "plr_execute_sharded": ([_P, _P, _P, _S, _I, _I, _P, _P], _st),
+    "plr_execute_host": ([_P, _P, _P, _S, _P], _st),
+    "plr_nccl_unique_id": ([_P, _S], _st),
+    "plr_nccl_comm_init": ([ctypes.POINTER(_P), _P, _I, _I], _st),
+    "plr_nccl_comm_destroy": ([_P], _st),
+    "plr_status_string": ([_I], ctypes.c_char_p),
+    "plr_last_error": ([], ctypes.c_char_p),
+    "plr_abi_version": ([], _I),
+}
+for _name, (_args, _res) in _SIGS.items():
+    _f = getattr(lib, _name)
+    _f.argtypes = _args
+    _f.restype = _res
+
+EXPORTED = tuple(_SIGS)
+
+_DTYPES = {"int32": 0, "float32": 1}
+_CLASSES = {0: "ONES", 1: "PERM", 2: "POLY", 3: "DECAY", 4: "FLOAT"}
+
+
+class PlanInfo(ctypes.Structure):
+    _fields_ = [("p", _I), ("k", _I), ("dtype", _I), ("cls", _I), ("elems_per_thread", _I),
+                ("threads_per_cta", _I), ("tile_elems", _I), ("stages", _I), ("decay_len", ctypes.c_int64),
+                ("fixup_len", ctypes.c_int64), ("n_max", _S), ("scratch_bytes", _S), ("ctas_per_sm", _I),
+                ("num_sms", _I)]
+
+
+class PLRError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        name = lib.plr_status_string(status).decode()
+        detail = lib.plr_last_error().decode()
+        super().__init__("%s: %s (%s)" % (where, name, detail))
+
+
+def _check(status: int, where: str):
+    if status != 0:
+        raise PLRError(status, where)
+
+
+def abi_version() -> int:
+    return lib.plr_abi_version()
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _stream_ptr(stream=None):
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _dev_ptr(t, dtype_name):
+    torch = _torch()
+    want = torch.int32 if dtype_name == "int32" else torch.float32
+    if not t.is_cuda:
+        raise ValueError("expected a CUDA tensor")
+    if t.dtype != want:
+        raise TypeError("expected %s, got %s" % (want, t.dtype))
+    if not t.is_contiguous():
+        raise ValueError("expected a contiguous tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def shard_bounds(n_total: int, world: int, rank: int):
+    """Contiguous rank-ordered segments (the last ranks get the remainder)."""
+    base, rem = divmod(n_total, world)
+    start = rank * base + max(0, rank - (world - rem))
+    return start, base + (1 if rank >= world - rem else 0)
+
+
+class Plan:
+    """A planned recurrence (signature a : b) for one dtype and up to n_max elements."""
+
+    def __init__(self, a, b, dtype: str = "int32", n_max: int = 1 << 30):
+        if dtype not in _DTYPES:
+            raise ValueError("dtype must be 'int32' or 'float32'")
+        self.a = tuple(float(v) for v in a)
+        self.b = tuple(float(v) for v in b)
+        self.dtype = dtype
+        self.p = len(self.a) - 1
+        self.k = len(self.b)
+        self.n_max = int(n_max)
+        arr_a = (ctypes.c_double * len(self.a))(*self.a)
+        arr_b = (ctypes.c_double * max(1, len(self.b)))(*self.b)
+        h = _P()
+        _check(lib.plr_plan_create(ctypes.byref(h), arr_a, self.p, arr_b, self.k, _DTYPES[dtype], self.n_max),
+               "plr_plan_create")
+        self._h = h
+        self._hist = None
+
+    # ------------------------------------------------------------------
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            lib.plr_plan_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    @property
+    def info(self) -> dict:
+        pi = PlanInfo()
+        _check(lib.plr_plan_get_info(self._h, ctypes.byref(pi)), "plr_plan_get_info")
+        d = {f: getattr(pi, f) for f, _ in PlanInfo._fields_}
+        d["cls"] = _CLASSES.get(d["cls"], str(d["cls"]))
+        d["dtype"] = "int32" if d["dtype"] == 0 else "float32"
+        return d
+
+    def factor_lists(self, m: int):
+        """The k seed-extended correction-factor lists (Sec. 2.1) as planned."""
+        import numpy as np
+        npdt = np.int32 if self.dtype == "int32" else np.float32
+        out = np.empty((self.k, self.k + m), dtype=npdt)
+        _check(lib.plr_plan_factor_lists(self._h, m, out.ctypes.data_as(_P)), "plr_plan_factor_lists")
+        return out
+
+    # ------------------------------------------------------------------
+    def _out(self, x, out):
+        torch = _torch()
+        if out is None:
+            out = torch.empty_like(x)
+        return out
+
+    def __call__(self, x, out=None, stream=None):
+        """y = recurrence(x) with zero initial conditions."""
+        out = self._out(x, out)
+        n = x.numel()
+        _check(lib.plr_execute(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), n, _stream_ptr(stream)),
+               "plr_execute")
+        return out
+
+    def continue_(self, x, out=None, x_hist=None, y_hist=None, stream=None):
+        """Continue a sequence from the p previous inputs and k previous outputs."""
+        out = self._out(x, out)
+        xh = _dev_ptr(x_hist, self.dtype) if x_hist is not None else None
+        yh = _dev_ptr(y_hist, self.dtype) if y_hist is not None else None
+        _check(lib.plr_execute_continue(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), x.numel(),
+                                        xh, yh, _stream_ptr(stream)), "plr_execute_continue")
+        return out
+
+    def reduce(self, x, payload=None, stream=None):
+        """Reduce-only pass: 64-byte end-state payload of x (zero history)."""
+        torch = _torch()
+        if payload is None:
+            payload = torch.empty(PAYLOAD_BYTES, dtype=torch.uint8, device=x.device)
+        _check(lib.plr_reduce(self._h, _dev_ptr(x, self.dtype), x.numel(), ctypes.c_void_p(payload.data_ptr()),
+                              _stream_ptr(stream)), "plr_reduce")
+        return payload
+
+    def payload_from_output(self, x, y, payload=None, stream=None):
+        torch = _torch()
+        if payload is None:
+            payload = torch.empty(PAYLOAD_BYTES, dtype=torch.uint8, device=x.device)
+        _check(lib.plr_payload_from_output(self._h, _dev_ptr(x, self.dtype), _dev_ptr(y, self.dtype), x.numel(),
+                                           ctypes.c_void_p(payload.data_ptr()), _stream_ptr(stream)),
+               "plr_payload_from_output")
+        return payload
+
+    def combine(self, payloads, rank: int, world: int, hist=None, stream=None):
+        """Boundary history of `rank` from all ranks' payloads (device)."""
+        torch = _torch()
+        if hist is None:
+            hist = torch.zeros(8, dtype=torch.int32, device=payloads.device)
+        _check(lib.plr_combine(self._h, ctypes.c_void_p(payloads.data_ptr()), rank, world,
+                               ctypes.c_void_p(hist.data_ptr()), _stream_ptr(stream)), "plr_combine")
+        return hist
+
+    def combine_host(self, payloads: bytes, rank: int, world: int) -> bytes:
+        """Same combine on the host (no GPU): payloads = world * 64 bytes."""
+        buf = ctypes.create_string_buffer(bytes(payloads), len(payloads))
+        hist = ctypes.create_string_buffer(32)
+        _check(lib.plr_combine_host(self._h, buf, rank, world, hist), "plr_combine_host")
+        return hist.raw
+
+    def fixup(self, y, hist, stream=None):
+        _check(lib.plr_fixup(self._h, _dev_ptr(y, self.dtype), y.numel(), ctypes.c_void_p(hist.data_ptr()),
+                             _stream_ptr(stream)), "plr_fixup")
+        return y
+
+    def execute_host(self, x_host, y_host=None, stream=None):
+        """End to end from host memory (pinned for full speed): chunked
+        H2D -> recurrence -> D2H with copies overlapped (synchronous)."""
+        torch = _torch()
+        if y_host is None:
+            y_host = torch.empty_like(x_host, pin_memory=x_host.is_pinned())
+        assert not x_host.is_cuda and not y_host.is_cuda
+        _check(lib.plr_execute_host(self._h, ctypes.c_void_p(x_host.data_ptr()), ctypes.c_void_p(y_host.data_ptr()),
+                                    x_host.numel(), _stream_ptr(stream)), "plr_execute_host")
+        return y_host
+
+    # ------------------------------------------------------------------
+    def sharded(self, x, out=None, comm: "ShardComm" = None, stream=None):
+        """This rank's contiguous segment of a sequence sharded over the
+        ranks of `comm` (one NCCL allgather of 64 bytes per rank)."""
+        out = self._out(x, out)
+        _check(lib.plr_execute_sharded(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), x.numel(),
+                                       comm.rank, comm.world, comm.handle, _stream_ptr(stream)),
+               "plr_execute_sharded")
+        return out
+
+
+class ShardComm:
+    """NCCL communicator of the library, bootstrapped through torch.distributed:
+    rank 0 creates the unique id, the process group broadcasts its bytes."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        idbuf = ctypes.create_string_buffer(128)
+        if self.rank == 0:
+            _check(lib.plr_nccl_unique_id(idbuf, 128), "plr_nccl_unique_id")
+        obj = [idbuf.raw if self.rank == 0 else None]
+        dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+        idbuf = ctypes.create_string_buffer(obj[0], 128)
+        h = _P()
+        _check(lib.plr_nccl_comm_init(ctypes.byref(h), idbuf, self.rank, self.world), "plr_nccl_comm_init")
+        self.handle = h
+
+    def close(self):
+        if self.handle is not None and self.handle.value:
+            lib.plr_nccl_comm_destroy(self.handle)
+            self.handle = None

@@ -1,0 +1,99 @@
+// plr_internal.h -- shared between the host planner, the kernels and the ABI.
+// Product code only; nothing here is shared with oracle/.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+
+#include "../../include/plr.h"
+
+namespace plr {
+
+// ---- kernel geometry -------------------------------------------------------
+// X contiguous elements per thread (odd: conflict-free strided shared-memory
+// access), W compute warps, S-stage shared-memory ring, plus one producer warp
+// that owns tickets, TMA bulk loads and TMA bulk stores.
+constexpr int kMaxK = PLR_MAX_K;
+constexpr int kMaxP = PLR_MAX_P;
+constexpr int kHalo = 4;            // words in front of each stage: x_{-4}..x_{-1}
+constexpr int kMaxX = 31;
+constexpr int kMaxW = 16;
+constexpr int kStatusWords = 4;     // u64 status words per tile (>= kMaxK)
+constexpr int kAug = 8;             // augmented state slots: x_{-4..-1}, y_{-4..-1}
+
+struct Geometry {
+    int X, W, S;
+    int tile() const { return 32 * W * X; }
+};
+
+// Transfer-matrix tables, row-major in a kMaxK x kMaxK slot.
+//   T(L)[q][r] = coefficient of S_r in S(s+L)_q, S(s) = (y_{s-1}, ..., y_{s-k}),
+// i.e. T(L) = M^L for the companion matrix M, and T(L)[q][r] = h^(r+1)_{L-1-q}
+// (the seed-extended correction factors of Sec. 2.1).
+template <typename T>
+struct Tables {
+    T alpha[kMaxP + 1];                  // a0, a-1, ..., a-p
+    T c[kMaxK];                          // b-1, ..., b-k
+    T H[kMaxX][kMaxK];                   // H[u][r] = h^(r+1)_u = T(u+1)[0][r], u < X
+    T Twarp[5][kMaxK * kMaxK];           // T(X * 2^s)          lane scan
+    T Tblk[4][kMaxK * kMaxK];            // T(32 X * 2^s)       warp-aggregate scan
+    T Twin[kMaxW][kMaxK * kMaxK];        // T(32 X * w)         warp carry-in
+    T Tlb[6][kMaxK * kMaxK];             // T(m * 2^s), s<=5    look-back fold
+};
+
+template <typename T>
+struct ScanParams {
+    const T* x;
+    T* y;
+    uint64_t n;
+    uint64_t ntiles;
+    unsigned long long ticket_base;
+    unsigned long long* ticket;
+    unsigned long long* status;          // ntiles x kStatusWords, {tag:32 | value:32}
+    uint32_t epoch;                      // tags 2*epoch (aggregate) / 2*epoch+1 (inclusive)
+    int decay;                           // T(m) == 0 exactly: inclusive == aggregate
+    const T* x_hist;                     // p values x_{-p}..x_{-1} or null
+    const T* y_hist;                     // k values y_{-k}..y_{-1} or null
+    T* y_tail;                           // k slots y_{n-k}..y_{n-1} or null
+    const T* lane_T;                     // [k*k][32]: T(X*l) per lane
+    Tables<T> tab;
+};
+
+// Host-side planner result.
+struct PlanTables {
+    int p, k;
+    plr_dtype dtype;
+    plr_class cls;
+    Geometry geo;
+    int64_t decay_len;
+    int64_t fixup_len;
+    int decay_flag;
+    Tables<uint32_t> ti;                 // int32 ring
+    Tables<float> tf;                    // fp32
+    uint32_t lane_i[kMaxK * kMaxK * 32];
+    float lane_f[kMaxK * kMaxK * 32];
+    // coefficients as the combine / fixup use them
+    double a_d[kMaxP + 1], b_d[kMaxK];
+    uint32_t a_u[kMaxP + 1], b_u[kMaxK];
+    // DECAY fixup: F[i][slot] = response of y_i to a unit in augmented slot
+    // (x_{-4..-1}, y_{-4..-1}) with zero input, i < fixup_len (fp32)
+    float* fix_table;                    // host, fixup_len * kAug (owned)
+};
+
+// planner (host, plr_planner.cpp)
+plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype dtype,
+                       Geometry geo, PlanTables* out, const char** why);
+void plan_tables_free(PlanTables* pt);
+void factor_lists(const PlanTables& pt, int64_t m, void* out);
+
+// 8x8 augmented companion matrix of Eq. (1) for the free evolution
+// (zero input) of the state (x_{-4..-1}, y_{-4..-1}); used by the combine.
+template <typename R>
+void aug_companion(const R* alpha, int p, const R* c, int k, R* M8) {
+    for (int i = 0; i < kAug * kAug; i++) M8[i] = R(0);
+    for (int i = 0; i < 3; i++) M8[i * kAug + (i + 1)] = R(1);        // x shift, x_{-1}' = 0
+    for (int i = 4; i < 7; i++) M8[i * kAug + (i + 1)] = R(1);        // y shift
+    for (int j = 1; j <= p; j++) M8[7 * kAug + (4 - j)] = alpha[j];   // y_new += a_{-j} x_{-j}
+    for (int j = 1; j <= k; j++) M8[7 * kAug + (8 - j)] = c[j - 1];   // y_new += b_{-j} y_{-j}
+}
+
+}  // namespace plr

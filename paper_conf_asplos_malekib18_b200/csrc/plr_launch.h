@@ -1,0 +1,42 @@
+// plr_launch.h -- host-side launch interface between the ABI and the
+// templated scan kernels (instantiated per dtype in plr_scan_{i32,f32}.cu).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "plr_internal.h"
+
+namespace plr {
+
+struct LaunchArgs {
+    const void* x;
+    void* y;
+    uint64_t n;
+    uint64_t ntiles;
+    unsigned long long ticket_base;
+    unsigned long long* ticket;
+    unsigned long long* status;
+    uint32_t epoch;
+    int decay;
+    const void* x_hist;
+    const void* y_hist;
+    void* y_tail;
+    const void* lane_T;
+    int grid;
+    bool store;
+    cudaStream_t stream;
+    int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel
+};
+
+// Tile geometry per dtype/order (must match an instantiated kernel).
+Geometry default_geometry(plr_dtype dtype, int k, int p);
+
+cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
+cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm);
+
+// per-dtype entry points
+cudaError_t launch_scan_i32(const PlanTables& pt, const LaunchArgs& la);
+cudaError_t launch_scan_f32(const PlanTables& pt, const LaunchArgs& la);
+cudaError_t occupancy_i32(const PlanTables& pt, int* ctas_per_sm);
+cudaError_t occupancy_f32(const PlanTables& pt, int* ctas_per_sm);
+
+}  // namespace plr

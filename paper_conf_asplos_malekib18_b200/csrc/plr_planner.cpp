@@ -1,0 +1,239 @@
+// plr_planner.cpp -- host-side planner of the PLR hot path (row a0 of
+// SURVEY.md §8(a)).
+//
+// The paper's generator checks the signature, computes the
+// correction factors as n-nacci numbers and emits them as k
+// constant arrays of m factors, with specialised code for
+// constant, 0/1, repeating and decaying factors.  Here the
+// planner computes, once per plan:
+//   * the companion matrix M of (1: c) and every transfer matrix
+//     T(L) = M^L the kernels need (repeated squaring; exact in Z/2^32, fp64
+//     then rounded to fp32 with denormals flushed for floats, SURVEY §7
+//     "Factor-table numerics");
+//   * the per-element factors h^(r)_u = T(u+1)[0][r-1] for u < x;
+//   * the class (ONES / PERM / POLY / DECAY / FLOAT) and, for DECAY, the
+//     last index at which the fp32 impulse response is nonzero (L_dec) and
+//     the free-response table used by the sharded fixup.
+#include <cmath>
+#include <cfloat>
+#include <cstdlib>
+#include <cstring>
+#include <vector>
+
+#include "plr_internal.h"
+
+namespace plr {
+namespace {
+
+// ---- small dense matrices over a ring --------------------------------------
+template <typename R>
+struct Mat {
+    int k;
+    R v[kMaxK * kMaxK];
+    explicit Mat(int k_ = 1) : k(k_) { for (auto& e : v) e = R(0); }
+    R& at(int q, int r) { return v[q * kMaxK + r]; }
+    R at(int q, int r) const { return v[q * kMaxK + r]; }
+    static Mat eye(int k) { Mat m(k); for (int i = 0; i < k; i++) m.at(i, i) = R(1); return m; }
+};
+
+template <typename R>
+Mat<R> mul(const Mat<R>& A, const Mat<R>& B) {
+    Mat<R> C(A.k);
+    for (int q = 0; q < A.k; q++)
+        for (int r = 0; r < A.k; r++) {
+            R acc = R(0);
+            for (int t = 0; t < A.k; t++) acc += A.at(q, t) * B.at(t, r);
+            C.at(q, r) = acc;
+        }
+    return C;
+}
+
+// companion matrix of the recurrence (1: c): S' = M S with
+// S = (y_{s-1}, ..., y_{s-k}) and zero input.
+template <typename R>
+Mat<R> companion(const R* c, int k) {
+    Mat<R> M(k);
+    for (int r = 0; r < k; r++) M.at(0, r) = c[r];
+    for (int q = 1; q < k; q++) M.at(q, q - 1) = R(1);
+    return M;
+}
+
+template <typename R>
+Mat<R> mpow(const Mat<R>& M, uint64_t L) {
+    Mat<R> result = Mat<R>::eye(M.k), base = M;
+    while (L) {
+        if (L & 1) result = mul(result, base);
+        L >>= 1;
+        if (L) base = mul(base, base);
+    }
+    return result;
+}
+
+inline float ftz(double v) {
+    float f = (float)v;
+    if (std::fabs(f) < FLT_MIN) f = 0.0f;       // flush denormals
+    return f;
+}
+
+template <typename R, typename T, typename Cvt>
+void store_mat(const Mat<R>& m, T* dst, Cvt cvt) {
+    for (int q = 0; q < kMaxK; q++)
+        for (int r = 0; r < kMaxK; r++)
+            dst[q * kMaxK + r] = (q < m.k && r < m.k) ? cvt(m.at(q, r)) : T(0);
+}
+
+template <typename R, typename T, typename Cvt>
+void fill_tables(const Mat<R>& M, int k, Geometry geo, Tables<T>* tb, T* lane, Cvt cvt) {
+    const uint64_t X = geo.X, m = (uint64_t)geo.tile();
+    for (int u = 0; u < kMaxX; u++) {
+        Mat<R> Tu = mpow(M, (uint64_t)u + 1);
+        for (int r = 0; r < kMaxK; r++) tb->H[u][r] = (u < geo.X && r < k) ? cvt(Tu.at(0, r)) : T(0);
+    }
+    for (int s = 0; s < 5; s++) store_mat(mpow(M, X << s), tb->Twarp[s], cvt);
+    for (int s = 0; s < 4; s++) store_mat(mpow(M, (32 * X) << s), tb->Tblk[s], cvt);
+    for (int w = 0; w < kMaxW; w++) store_mat(mpow(M, 32 * X * (uint64_t)w), tb->Twin[w], cvt);
+    for (int s = 0; s < 6; s++) store_mat(mpow(M, m << s), tb->Tlb[s], cvt);
+    for (int l = 0; l < 32; l++) {
+        Mat<R> Tl = mpow(M, X * (uint64_t)l);
+        for (int q = 0; q < k; q++)
+            for (int r = 0; r < k; r++) lane[(q * k + r) * 32 + l] = cvt(Tl.at(q, r));
+    }
+}
+
+}  // namespace
+
+plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype dtype,
+                       Geometry geo, PlanTables* out, const char** why) {
+    *why = "";
+    if (a == nullptr || b == nullptr || out == nullptr) { *why = "null argument"; return PLR_ERR_INVALID_ARG; }
+    if (dtype != PLR_INT32 && dtype != PLR_FLOAT32) { *why = "dtype must be PLR_INT32 or PLR_FLOAT32"; return PLR_ERR_DTYPE; }
+    if (k < 1) { *why = "order k must be >= 1 (P:89-93)"; return PLR_ERR_SIGNATURE; }
+    if (p < 0) { *why = "p must be >= 0"; return PLR_ERR_SIGNATURE; }
+    if (k > kMaxK || p > kMaxP) { *why = "k > PLR_MAX_K or p > PLR_MAX_P"; return PLR_ERR_SIZE; }
+    for (int j = 0; j <= p; j++) if (!std::isfinite(a[j])) { *why = "non-finite coefficient"; return PLR_ERR_SIGNATURE; }
+    for (int j = 0; j < k; j++) if (!std::isfinite(b[j])) { *why = "non-finite coefficient"; return PLR_ERR_SIGNATURE; }
+    if (a[p] == 0.0) { *why = "last non-recursive coefficient must not be zero (P:635-637)"; return PLR_ERR_SIGNATURE; }
+    if (b[k - 1] == 0.0) { *why = "last recursive coefficient must not be zero (P:635-637)"; return PLR_ERR_SIGNATURE; }
+    if (dtype == PLR_INT32) {
+        for (int j = 0; j <= p + k; j++) {
+            double v = j <= p ? a[j] : b[j - p - 1];
+            if (v != std::floor(v) || v < -2147483648.0 || v >= 4294967296.0) {
+                *why = "PLR_INT32 needs integer coefficients in [-2^31, 2^32)";
+                return PLR_ERR_SIGNATURE;
+            }
+        }
+    } else {
+        for (int j = 0; j <= p + k; j++) {
+            double v = j <= p ? a[j] : b[j - p - 1];
+            if (std::fabs(v) > FLT_MAX) { *why = "coefficient overflows fp32"; return PLR_ERR_SIGNATURE; }
+        }
+        if ((float)a[p] == 0.0f || (float)b[k - 1] == 0.0f) { *why = "last coefficient rounds to 0 in fp32"; return PLR_ERR_SIGNATURE; }
+    }
+    if (geo.X < k || geo.X > kMaxX || geo.W > kMaxW || (geo.W & (geo.W - 1))) { *why = "bad geometry"; return PLR_ERR_INVALID_ARG; }
+
+    PlanTables& pt = *out;
+    std::memset(&pt, 0, sizeof(pt));
+    pt.p = p; pt.k = k; pt.dtype = dtype; pt.geo = geo;
+    pt.decay_len = -1; pt.fixup_len = 0;
+    pt.fix_table = nullptr;
+
+    if (dtype == PLR_INT32) {
+        uint32_t c[kMaxK] = {0};
+        for (int j = 0; j <= p; j++) pt.a_u[j] = (uint32_t)(int64_t)(a[j] < 0 ? a[j] : std::fmod(a[j], 4294967296.0));
+        for (int j = 0; j < k; j++) c[j] = pt.b_u[j] = (uint32_t)(int64_t)(b[j] < 0 ? b[j] : std::fmod(b[j], 4294967296.0));
+        for (int j = 0; j <= kMaxP; j++) pt.ti.alpha[j] = j <= p ? pt.a_u[j] : 0u;
+        for (int j = 0; j < kMaxK; j++) pt.ti.c[j] = j < k ? c[j] : 0u;
+        Mat<uint32_t> M = companion<uint32_t>(c, k);
+        fill_tables(M, k, geo, &pt.ti, pt.lane_i, [](uint32_t v) { return v; });
+        // class: all factors 1 -> ONES; single unit feedback
+        // coefficient -> PERM (0/1 repeating factors); otherwise POLY
+        int nnz = 0, ones = 0;
+        for (int j = 0; j < k; j++) { nnz += c[j] != 0; ones += c[j] == 1u; }
+        if (k == 1 && c[0] == 1u) pt.cls = PLR_CLASS_ONES;
+        else if (nnz == 1 && ones == 1) pt.cls = PLR_CLASS_PERM;
+        else pt.cls = PLR_CLASS_POLY;
+        pt.decay_flag = 0;
+    } else {
+        double c[kMaxK] = {0}, al[kMaxP + 1] = {0};
+        for (int j = 0; j <= p; j++) al[j] = pt.a_d[j] = (double)(float)a[j];
+        for (int j = 0; j < k; j++) c[j] = pt.b_d[j] = (double)(float)b[j];
+        for (int j = 0; j <= kMaxP; j++) pt.tf.alpha[j] = j <= p ? (float)al[j] : 0.0f;
+        for (int j = 0; j < kMaxK; j++) pt.tf.c[j] = j < k ? (float)c[j] : 0.0f;
+        Mat<double> M = companion<double>(c, k);
+        fill_tables(M, k, geo, &pt.tf, pt.lane_f, [](double v) { return ftz(v); });
+        // DECAY: the fp32 impulse response g of (1: c) becomes
+        // exactly 0 and stays 0.  g_0 = 1, g_u = sum_j c_j g_{u-j}.
+        const int64_t cap = 1 << 16;
+        std::vector<double> g(cap, 0.0);
+        int64_t last = -1;
+        for (int64_t u = 0; u < cap; u++) {
+            double v = (u == 0) ? 1.0 : 0.0;
+            for (int j = 1; j <= k; j++) if (u - j >= 0) v += c[j - 1] * g[u - j];
+            g[u] = v;
+            if (ftz(v) != 0.0f) last = u;
+        }
+        const bool decays = last < cap / 2;
+        bool tm_zero = true;
+        for (int e = 0; e < kMaxK * kMaxK; e++) tm_zero = tm_zero && pt.tf.Tlb[0][e] == 0.0f;
+        pt.decay_flag = (decays && tm_zero) ? 1 : 0;
+        pt.cls = decays ? PLR_CLASS_DECAY : PLR_CLASS_FLOAT;
+        if (decays) {
+            pt.decay_len = last;
+            // free response of the augmented state (x_{-4..-1}, y_{-4..-1})
+            std::vector<double> F((size_t)cap * kAug, 0.0);
+            int64_t lastf = -1;
+            for (int slot = 0; slot < kAug; slot++) {
+                std::vector<double> xs(4, 0.0), ys(4, 0.0);
+                if (slot < 4) xs[slot] = 1.0; else ys[slot - 4] = 1.0;
+                std::vector<double> y(cap, 0.0);
+                for (int64_t i = 0; i < cap; i++) {
+                    double v = 0.0;
+                    for (int j = 1; j <= p; j++) v += al[j] * (i - j >= 0 ? 0.0 : xs[4 + (i - j)]);
+                    for (int j = 1; j <= k; j++) v += c[j - 1] * (i - j >= 0 ? y[i - j] : ys[4 + (i - j)]);
+                    y[i] = v;
+                    F[(size_t)i * kAug + slot] = v;
+                    if (ftz(v) != 0.0f && i > lastf) lastf = i;
+                }
+            }
+            pt.fixup_len = lastf + 1;
+            pt.fix_table = (float*)std::malloc(sizeof(float) * (size_t)(pt.fixup_len > 0 ? pt.fixup_len : 1) * kAug);
+            for (int64_t i = 0; i < pt.fixup_len; i++)
+                for (int s = 0; s < kAug; s++) pt.fix_table[i * kAug + s] = ftz(F[(size_t)i * kAug + s]);
+        }
+    }
+    return PLR_OK;
+}
+
+void plan_tables_free(PlanTables* pt) {
+    if (pt && pt->fix_table) { std::free(pt->fix_table); pt->fix_table = nullptr; }
+}
+
+// k rows of (k + m): seed in memory order w_{m-k}..w_{m-1} (a one at the
+// carry's position), then h^(r)_u = T(u+1)[0][r-1], u < m, from
+// the same matrix powers the kernel tables come from.
+void factor_lists(const PlanTables& pt, int64_t m, void* out) {
+    const int k = pt.k;
+    const int64_t len = k + m;
+    if (pt.dtype == PLR_INT32) {
+        uint32_t* o = (uint32_t*)out;
+        Mat<uint32_t> M = companion<uint32_t>(pt.ti.c, k);
+        for (int r = 1; r <= k; r++)
+            for (int q = 0; q < k; q++) o[(r - 1) * len + q] = (q == k - r) ? 1u : 0u;
+        Mat<uint32_t> Tu = Mat<uint32_t>::eye(k);
+        for (int64_t u = 0; u < m; u++) {
+            Tu = mpow(M, (uint64_t)u + 1);
+            for (int r = 1; r <= k; r++) o[(r - 1) * len + k + u] = Tu.at(0, r - 1);
+        }
+    } else {
+        float* o = (float*)out;
+        Mat<double> M = companion<double>(pt.b_d, k);
+        for (int r = 1; r <= k; r++)
+            for (int q = 0; q < k; q++) o[(r - 1) * len + q] = (q == k - r) ? 1.0f : 0.0f;
+        for (int64_t u = 0; u < m; u++) {
+            Mat<double> Tu = mpow(M, (uint64_t)u + 1);
+            for (int r = 1; r <= k; r++) o[(r - 1) * len + k + u] = ftz(Tu.at(0, r - 1));
+        }
+    }
+}
+
+}  // namespace plr

@@ -1,0 +1,136 @@
+"""C-ABI checks that need no GPU: the library loads, exports every symbol of
+include/plr.h, validates signatures, and its host-side
+planner reproduces the paper's correction factors (worked example
+P:584-586, n-nacci P:350-361) against the independent oracle."""
+import ctypes
+import re
+import struct
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+from conftest import ROOT, read_golden
+
+plr = pytest.importorskip("paper_conf_asplos_malekib18_b200")
+
+
+def header_symbols():
+    src = open(ROOT + "/include/plr.h").read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(plr_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_exports_every_declared_symbol():
+    syms = header_symbols()
+    assert len(syms) >= 18
+    for s in syms:
+        assert hasattr(plr.lib, s), s
+    assert set(syms) == set(plr.binding.EXPORTED)
+    assert plr.abi_version() == 1
+
+
+@pytest.mark.parametrize("a,b,dtype,code", [
+    ((1,), (), "int32", 2),                 # k = 0: a map, excluded
+    ((0,), (1,), "int32", 2),               # last non-recursive coefficient 0
+    ((1,), (1, 0), "int32", 2),             # trailing zero feedback coefficient
+    ((1, 0), (1,), "int32", 2),             # trailing zero feed-forward coefficient
+    ((1.5,), (1,), "int32", 2),             # non-integer for PLR_INT32
+    ((1,), (1, 1, 1, 1, 1), "int32", 4),    # k > PLR_MAX_K
+    ((1, 1, 1, 1, 1), (1,), "float32", 4),  # p > PLR_MAX_P
+    ((float("nan"),), (0.5,), "float32", 2),
+])
+def test_signature_validation(a, b, dtype, code):
+    with pytest.raises(plr.PLRError) as e:
+        plr.Plan(a, b, dtype, n_max=0)
+    assert e.value.status == code
+
+
+def test_classes():
+    cls = {s.name: plr.Plan(s.a, s.b, s.dtype, n_max=0).info["cls"] for s in workloads.TABLE1}
+    assert cls["prefix"] == "ONES"
+    assert cls["tuple2"] == cls["tuple3"] == "PERM"
+    assert cls["order2"] == cls["order3"] == "POLY"
+    for nm in ("lp1", "lp2", "lp3", "hp1", "hp2", "hp3"):
+        assert cls[nm] == "DECAY"
+    assert plr.Plan((1.0,), (1.0,), "float32", n_max=0).info["cls"] == "FLOAT"
+
+
+def test_decay_length_matches_ftz_threshold():
+    """(1: 0.8): g_u = 0.8^u (fp32 coefficient) drops below FLT_MIN, where it
+    is flushed, after u = floor(log(FLT_MIN)/log(c))."""
+    c = float(np.float32(0.8))
+    expect = int(np.floor(np.log(np.finfo(np.float32).tiny) / np.log(c)))
+    assert plr.Plan((0.2,), (0.8,), "float32", n_max=0).info["decay_len"] == expect
+
+
+def test_planner_factor_lists_worked_example():
+    g = read_golden("worked_example.txt")
+    L = plr.Plan((1,), (2, -1), "int32", n_max=0).factor_lists(8)
+    assert L[0].tolist() == g["list1"] and L[1].tolist() == g["list2"]
+
+
+def test_planner_factor_lists_nnacci():
+    o = read_golden("nnacci.txt")
+    L = plr.Plan((1,), (1, 1, 1), "int32", n_max=0).factor_lists(17)
+    assert L[0].tolist() == o["A000073"][:20]
+    assert L[1].tolist() == o["A001590"][:20]
+    assert L[2].tolist() == [1] + o["A000073"][:19]
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+def test_planner_factor_lists_vs_oracle(sig):
+    """Planner (matrix powers) vs oracle (n-nacci iteration) over 600 factors."""
+    m = 600
+    L = plr.Plan(sig.a, sig.b, sig.dtype, n_max=0).factor_lists(m)
+    ref = oracle.factor_lists(sig.b, m, sig.dtype)
+    if sig.dtype == "int32":
+        assert np.array_equal(L, ref)
+    else:
+        r32 = ref.astype(np.float32)
+        r32[np.abs(r32) < np.finfo(np.float32).tiny] = 0           # FTZ
+        np.testing.assert_allclose(L, r32, rtol=2e-6, atol=0)
+
+
+def _payload(n, x_tail, y_tail, dtype):
+    npdt = np.int32 if dtype == "int32" else np.float32
+    xt = np.zeros(4, npdt)
+    yt = np.zeros(4, npdt)
+    if len(x_tail):
+        xt[4 - len(x_tail):] = x_tail
+    if len(y_tail):
+        yt[4 - len(y_tail):] = y_tail
+    return struct.pack("<Q", n) + xt.tobytes() + yt.tobytes() + bytes(24)
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+def test_combine_host_matches_oracle(sig):
+    """The segment prefix z_{r+1} = M^{n_r} z_r + payload_r reproduces the
+    true boundary history (reading R12) for uneven segments, incl. n_r < k."""
+    sizes = [5000, 3, 1777, 0, 4096, 1]
+    x = workloads.host_input(sum(sizes), sig.dtype, 11)
+    yfull = oracle.recurrence(x, sig.a, sig.b, sig.dtype)
+    plan = plr.Plan(sig.a, sig.b, sig.dtype, n_max=0)
+    pls = b""
+    off = 0
+    for nr in sizes:
+        seg = x[off:off + nr]
+        yz = oracle.recurrence(seg, sig.a, sig.b, sig.dtype)     # zero history
+        if sig.dtype == "float32":
+            yz = yz.astype(np.float32)
+        pls += _payload(nr, seg[-4:] if nr else [], yz[-4:] if nr else [], sig.dtype)
+        off += nr
+    starts = np.cumsum([0] + sizes)
+    for r in range(len(sizes)):
+        hist = plan.combine_host(pls, r, len(sizes))
+        npdt = np.int32 if sig.dtype == "int32" else np.float32
+        h = np.frombuffer(hist, dtype=npdt)
+        s = starts[r]
+        ex_x = np.array([x[s - 4 + i] if s - 4 + i >= 0 else 0 for i in range(4)], dtype=npdt)
+        ex_y = np.array([yfull[s - 4 + i] if s - 4 + i >= 0 else 0 for i in range(4)])
+        assert np.array_equal(h[:4], ex_x)
+        if sig.dtype == "int32":
+            assert np.array_equal(h[4:], ex_y.astype(np.int32))
+        else:
+            np.testing.assert_allclose(h[4:], ex_y, rtol=1e-5, atol=1e-5)

@@ -1,0 +1,261 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle, element by
+element, on seeded inputs.  Bar: bit-exact for int32
+(ring Z/2^32); for float32 max_i |y_gpu - y_ref| / max(1, |y_ref|) <= 1e-4
+against the fp64 oracle (BASELINE.json north_star; the paper used 1e-3
+against serial fp32)."""
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-4
+M = 3840                 # tile of the default geometry (checked below)
+
+
+def rel_err(y, ref):
+    y = np.asarray(y, dtype=np.float64)
+    return float(np.max(np.abs(y - ref) / np.maximum(1.0, np.abs(ref)))) if len(ref) else 0.0
+
+
+def check(y, ref, dtype, what=""):
+    if dtype == "int32":
+        bad = np.flatnonzero(y != ref)
+        assert bad.size == 0, "%s: %d mismatches, first at %d: %d vs %d" % (
+            what, bad.size, bad[0], y[bad[0]], ref[bad[0]])
+    else:
+        e = rel_err(y, ref)
+        assert e <= TOL, "%s: rel err %.3g" % (what, e)
+
+
+def run(plr, torch, sig, x, n_max=None):
+    plan = plr.Plan(sig.a, sig.b, sig.dtype, n_max=n_max or max(1, len(x)))
+    xd = torch.from_numpy(x).cuda()
+    y = plan(xd).cpu().numpy()
+    plan.close()
+    return y
+
+
+SIZES = [1, 2, 3, 4, 5, 14, 15, 16, 31, 32, 33, 480, 481, M - 1, M, M + 1, 3 * M + 7, 33 * M + 5,
+         (1 << 16) + 3, (1 << 20) + 12345]
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+def test_parity_sizes(cuda_plr, sig):
+    import torch
+    info = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 10).info
+    assert info["tile_elems"] == M
+    x_all = workloads.host_input(max(SIZES), sig.dtype, workloads.seed_for(1))
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=max(SIZES))
+    for n in SIZES:
+        x = x_all[:n].copy()
+        y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+        check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s n=%d" % (sig.name, n))
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+@pytest.mark.parametrize("kind", ["ones", "impulse", "alternating", "extremes"])
+def test_parity_structured(cuda_plr, sig, kind):
+    import torch
+    n = 7 * M + 123
+    x = workloads.structured_input(kind, n, sig.dtype)
+    y = run(cuda_plr, torch, sig, x)
+    check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s %s" % (sig.name, kind))
+
+
+def test_worked_example_on_gpu(cuda_plr):
+    import torch
+    from conftest import read_golden
+    g = read_golden("worked_example.txt")
+    x = np.array(g["input"], dtype=np.int32)
+    y = run(cuda_plr, torch, workloads.BY_NAME["order2"], x)
+    assert y.tolist() == g["expected_output"]
+
+
+def test_closed_forms_on_gpu(cuda_plr):
+    """ones -> i+1, C(i+2,2), C(i+3,3) mod 2^32 across ~270 tiles."""
+    import torch
+    n = (1 << 20) + 77
+    i = np.arange(n, dtype=np.uint64)
+    x = np.ones(n, dtype=np.int32)
+    for b, e in (((1,), i + 1), ((2, -1), (i + 1) * (i + 2) // 2), ((3, -3, 1), (i + 1) * (i + 2) * (i + 3) // 6)):
+        sig = workloads.Signature("t", (1,), b, "int32", "", "")
+        y = run(cuda_plr, torch, sig, x)
+        assert np.array_equal(y.view(np.uint32), (e % (1 << 32)).astype(np.uint32))
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+def test_repeated_launches_epochs(cuda_plr, sig):
+    """One plan, many launches with varying n: epoch-tagged status words and
+    the ticket base must never mix launches."""
+    import torch
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=200 * M)
+    rng = np.random.default_rng(5)
+    for t in range(12):
+        n = int(rng.integers(1, 200 * M))
+        x = workloads.host_input(n, sig.dtype, 100 + t)
+        y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+        check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s launch %d n=%d" % (sig.name, t, n))
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+def test_continue_chunks(cuda_plr, sig):
+    """plr_execute_continue over chunks (history = preceding inputs/outputs)
+    equals one call (P:78 zero state only at the very start)."""
+    import torch
+    n = 50 * M + 999
+    x = workloads.host_input(n, sig.dtype, 21)
+    ref = oracle.recurrence(x, sig.a, sig.b, sig.dtype)
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    xd = torch.from_numpy(x).cuda()
+    yd = torch.empty_like(xd)
+    cuts = [0, 5, 4096, 4100, 20 * M + 8, 20 * M + 12, n]
+    for s, e in zip(cuts[:-1], cuts[1:]):
+        xh = xd[s - sig.p:s] if (sig.p and s >= sig.p) else None
+        yh = yd[s - sig.k:s] if s >= sig.k else None
+        if s > 0 and (xh is None and sig.p) or (s > 0 and yh is None):
+            # histories that reach before index 0: pad with zeros
+            xh = torch.cat([torch.zeros(max(0, sig.p - s), dtype=xd.dtype, device="cuda"), xd[max(0, s - sig.p):s]]) if sig.p else None
+            yh = torch.cat([torch.zeros(max(0, sig.k - s), dtype=xd.dtype, device="cuda"), yd[max(0, s - sig.k):s]])
+        if s == 0:
+            xh, yh = None, None
+        plan.continue_(xd[s:e], yd[s:e], x_hist=xh, y_hist=yh)
+    check(yd.cpu().numpy(), ref, sig.dtype, sig.name)
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+def test_reduce_payload_and_combine(cuda_plr, sig):
+    """Reduce-only payload = zero-history end state; device combine = host
+    combine; and the full loopback of the sharded schedule on one GPU
+    (reduce or local pass -> gathered payloads -> combine -> seeded pass or
+    DECAY fixup) reproduces the oracle over the concatenation (reading R12)."""
+    import torch
+    sizes = [7 * M + 5, 3, 12 * M, M - 1, 9 * M + 1000]
+    n = sum(sizes)
+    x = workloads.host_input(n, sig.dtype, 31)
+    ref = oracle.recurrence(x, sig.a, sig.b, sig.dtype)
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    decay = plan.info["cls"] == "DECAY"
+    xd = torch.from_numpy(x).cuda()
+    yd = torch.empty_like(xd)
+    starts = np.cumsum([0] + sizes)
+    pls = []
+    for r, nr in enumerate(sizes):
+        seg = xd[starts[r]:starts[r] + nr]
+        if decay:
+            plan(seg, yd[starts[r]:starts[r] + nr])
+            pl = plan.payload_from_output(seg, yd[starts[r]:starts[r] + nr])
+        else:
+            pl = plan.reduce(seg)
+        # payload == oracle zero-history tails
+        yz = oracle.recurrence(x[starts[r]:starts[r] + nr], sig.a, sig.b, sig.dtype)
+        got = pl.cpu().numpy()
+        assert int(got[:8].view(np.uint64)[0]) == nr
+        npdt = np.int32 if sig.dtype == "int32" else np.float32
+        yt = got[24:40].view(npdt)[4 - min(4, nr):]
+        check(yt.astype(np.float64) if sig.dtype == "float32" else yt, yz[-4:], sig.dtype, "payload %d" % r)
+        pls.append(pl)
+    payloads = torch.cat(pls)
+    host_pl = payloads.cpu().numpy().tobytes()
+    for r, nr in enumerate(sizes):
+        hist = plan.combine(payloads, r, len(sizes))
+        assert hist.cpu().numpy().tobytes() == plan.combine_host(host_pl, r, len(sizes))
+        seg = xd[starts[r]:starts[r] + nr]
+        out = yd[starts[r]:starts[r] + nr]
+        if decay:
+            plan.fixup(out, hist)
+        else:
+            xh = hist[4 - sig.p:4] if sig.p else None
+            plan.continue_(seg, out, x_hist=xh, y_hist=hist[8 - sig.k:8])
+    check(yd.cpu().numpy(), ref, sig.dtype, sig.name)
+
+
+@pytest.mark.parametrize("sig", [workloads.BY_NAME[n] for n in ("prefix", "order3", "hp3")], ids=lambda s: s.name)
+def test_execute_sharded_world1(cuda_plr, sig):
+    import torch
+    n = 40 * M + 17
+    x = workloads.host_input(n, sig.dtype, 41)
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+
+    class C:
+        rank, world, handle = 0, 1, None
+    y = plan.sharded(torch.from_numpy(x).cuda(), comm=C()).cpu().numpy()
+    check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, sig.name)
+
+
+@pytest.mark.parametrize("sig", [workloads.BY_NAME[n] for n in ("tuple3", "lp2")], ids=lambda s: s.name)
+def test_execute_host_pipeline(cuda_plr, sig):
+    """plr_execute_host: chunked H2D/compute/D2H, chunks continued."""
+    import torch
+    n = (1 << 26) + 3 * M + 11              # > 2 chunks of 2^25
+    x = workloads.host_input(n, sig.dtype, 51)
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    xh = torch.from_numpy(x).pin_memory()
+    y = plan.execute_host(xh).numpy()
+    check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, sig.name)
+
+
+def test_errors(cuda_plr):
+    import torch
+    plan = cuda_plr.Plan((1, 1), (0.5,), "float32", n_max=1000)
+    x = torch.zeros(1000, dtype=torch.float32, device="cuda")
+    with pytest.raises(cuda_plr.PLRError) as e:
+        plan(x, x)                               # p > 0 in place
+    assert e.value.status == 5
+    with pytest.raises(cuda_plr.PLRError) as e:
+        plan(x[1:], torch.empty(999, device="cuda"))
+    assert e.value.status == 6                   # misaligned
+    big = torch.zeros(1001, dtype=torch.float32, device="cuda")
+    with pytest.raises(cuda_plr.PLRError) as e:
+        plan(big)
+    assert e.value.status == 4
+    plan2 = cuda_plr.Plan((1,), (1,), "int32", n_max=1000)
+    xi = torch.arange(1000, dtype=torch.int32, device="cuda")
+    ref = oracle.recurrence(xi.cpu().numpy(), (1,), (1,), "int32")
+    assert np.array_equal(plan2(xi, xi).cpu().numpy(), ref)   # p == 0 in place is allowed
+    assert plan2(torch.zeros(0, dtype=torch.int32, device="cuda")).numel() == 0
+
+
+# ------------------------------------------------------------ full size ----
+FULL = 1 << 30
+
+
+def _stream_check(plr_mod, torch, sig, n, seed, seg=1 << 25):
+    """Full-size run in the bench's launch configuration; the oracle streams
+    over segments with its history carried (O(segment) host memory) and every
+    output element is compared."""
+    plan = plr_mod.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    xd = workloads.device_input(n, sig.dtype, seed)
+    yd = plan(xd)
+    torch.cuda.synchronize()
+    xh = yh = None
+    worst = 0.0
+    for s in range(0, n, seg):
+        e = min(n, s + seg)
+        x = xd[s:e].cpu().numpy()
+        y = yd[s:e].cpu().numpy()
+        ref = oracle.recurrence(x, sig.a, sig.b, sig.dtype, x_hist=xh, y_hist=yh)
+        if sig.dtype == "int32":
+            assert np.array_equal(y, ref), "%s mismatch in [%d, %d)" % (sig.name, s, e)
+        else:
+            worst = max(worst, rel_err(y, ref))
+        xh = x[len(x) - sig.p:] if sig.p else None
+        yh = ref[len(ref) - sig.k:]
+    assert worst <= TOL, (sig.name, worst)
+    del xd, yd
+    plan.close()
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("name", ["tuple2", "tuple3", "order2", "order3", "lp1", "lp2", "hp2", "prefix"])
+def test_full_size_parity(cuda_plr, name):
+    import torch
+    sig = workloads.BY_NAME[name]
+    _stream_check(cuda_plr, torch, sig, FULL, workloads.seed_for(2))
+
+
+def test_full_size_ragged(cuda_plr):
+    import torch
+    _stream_check(cuda_plr, torch, workloads.BY_NAME["hp3"], FULL - 12345, workloads.seed_for(6))
