@@ -1,4 +1,4 @@
-// plr_dispatch.cu -- dtype dispatch and tile geometry.
+// plr_dispatch.cu -- dtype / accumulation dispatch and tile geometry.
 #include "plr_launch.h"
 
 namespace plr {
@@ -10,11 +10,16 @@ Geometry default_geometry(plr_dtype, int, int) {
 }
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la) {
-    return pt.dtype == PLR_INT32 ? launch_scan_i32(pt, la) : launch_scan_f32(pt, la);
+    if (pt.dtype == PLR_INT32) return launch_scan_i32(pt.ti, la, pt.k, pt.p);
+    if (pt.acc64) return launch_scan_f64acc(pt.td, la, pt.k, pt.p);
+    return launch_scan_f32(pt.tf, la, pt.k, pt.p);
 }
 
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm) {
-    return pt.dtype == PLR_INT32 ? occupancy_i32(pt, ctas_per_sm) : occupancy_f32(pt, ctas_per_sm);
+    LaunchArgs la{};
+    la.store = true;
+    la.occupancy_out = ctas_per_sm;
+    return launch_scan(pt, la);
 }
 
 }  // namespace plr

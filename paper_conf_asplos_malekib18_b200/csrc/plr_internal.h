@@ -11,7 +11,7 @@ namespace plr {
 // ---- kernel geometry -------------------------------------------------------
 // X contiguous elements per thread (odd: conflict-free strided shared-memory
 // access), W compute warps, S-stage shared-memory ring, plus one producer warp
-// that owns tickets, TMA bulk loads and TMA bulk stores.
+// (tickets, TMA bulk loads/stores) and one look-back warp.
 constexpr int kMaxK = PLR_MAX_K;
 constexpr int kMaxP = PLR_MAX_P;
 constexpr int kHalo = 4;            // words in front of each stage: x_{-4}..x_{-1}
@@ -19,28 +19,35 @@ constexpr int kMaxX = 31;
 constexpr int kMaxW = 16;
 constexpr int kStatusWords = 4;     // u64 status words per tile (>= kMaxK)
 constexpr int kAug = 8;             // augmented state slots: x_{-4..-1}, y_{-4..-1}
+constexpr int kTPL = 8;             // look-back: tiles per lane in a wide window
 
 struct Geometry {
     int X, W, S;
     int tile() const { return 32 * W * X; }
 };
 
-// Transfer-matrix tables, row-major in a kMaxK x kMaxK slot.
+// Tables the scan kernel reads from its parameter space.  T is the data type
+// (uint32_t ring or float), A the accumulation type of the local recurrence
+// and of every carry (uint32_t, float or double; see plan_tables()).
 //   T(L)[q][r] = coefficient of S_r in S(s+L)_q, S(s) = (y_{s-1}, ..., y_{s-k}),
 // i.e. T(L) = M^L for the companion matrix M, and T(L)[q][r] = h^(r+1)_{L-1-q}
 // (the seed-extended correction factors of Sec. 2.1).
-template <typename T>
+template <typename T, typename A>
 struct Tables {
-    T alpha[kMaxP + 1];                  // a0, a-1, ..., a-p
-    T c[kMaxK];                          // b-1, ..., b-k
+    T alpha[kMaxP + 1];                  // a0, a-1, ..., a-p       (FIR, data type)
+    A c[kMaxK];                          // b-1, ..., b-k           (recurrence)
     T H[kMaxX][kMaxK];                   // H[u][r] = h^(r+1)_u = T(u+1)[0][r], u < X
-    T Twarp[5][kMaxK * kMaxK];           // T(X * 2^s)          lane scan
-    T Tblk[4][kMaxK * kMaxK];            // T(32 X * 2^s)       warp-aggregate scan
-    T Twin[kMaxW][kMaxK * kMaxK];        // T(32 X * w)         warp carry-in
-    T Tlb[6][kMaxK * kMaxK];             // T(m * 2^s), s<=5    look-back fold
+    A Twarp[5][kMaxK * kMaxK];           // T(X * 2^s)          lane scan
+    A Tblk[4][kMaxK * kMaxK];            // T(32 X * 2^s)       warp-aggregate scan
+    A Twin[kMaxW][kMaxK * kMaxK];        // T(32 X * w)         warp carry-in
+    A Tm[kMaxK * kMaxK];                 // T(m)                inclusive = agg + T(m) G
+    A Tlb1[5][kMaxK * kMaxK];            // T(m * 2^s)          narrow window fold
+    A Tlb8[5][kMaxK * kMaxK];            // T(kTPL m * 2^s)     wide window fold
+    A Tw1[kMaxK * kMaxK];                // T(32 m)             next narrow window
+    A Tw8[kMaxK * kMaxK];                // T(32 kTPL m)        next wide window
 };
 
-template <typename T>
+template <typename T, typename A>
 struct ScanParams {
     const T* x;
     T* y;
@@ -54,8 +61,8 @@ struct ScanParams {
     const T* x_hist;                     // p values x_{-p}..x_{-1} or null
     const T* y_hist;                     // k values y_{-k}..y_{-1} or null
     T* y_tail;                           // k slots y_{n-k}..y_{n-1} or null
-    const T* lane_T;                     // [k*k][32]: T(X*l) per lane
-    Tables<T> tab;
+    const A* lane_T;                     // [k*k][32]: T(X*l) per lane
+    Tables<T, A> tab;
 };
 
 // Host-side planner result.
@@ -67,10 +74,14 @@ struct PlanTables {
     int64_t decay_len;
     int64_t fixup_len;
     int decay_flag;
-    Tables<uint32_t> ti;                 // int32 ring
-    Tables<float> tf;                    // fp32
+    int acc64;                           // float: accumulate recurrence + carries in fp64
+    double cond_bound;                   // eps32 * sum|a| * (sum|g|)^2 (float)
+    Tables<uint32_t, uint32_t> ti;       // int32 ring
+    Tables<float, float> tf;             // fp32, fp32 accumulation
+    Tables<float, double> td;            // fp32, fp64 accumulation
     uint32_t lane_i[kMaxK * kMaxK * 32];
     float lane_f[kMaxK * kMaxK * 32];
+    double lane_d[kMaxK * kMaxK * 32];
     // coefficients as the combine / fixup use them
     double a_d[kMaxP + 1], b_d[kMaxK];
     uint32_t a_u[kMaxP + 1], b_u[kMaxK];

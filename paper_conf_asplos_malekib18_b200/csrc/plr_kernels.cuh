@@ -1,23 +1,27 @@
 // plr_kernels.cuh -- sm_100a kernels of the PLR hot path.
 //
-// One persistent single-pass kernel evaluates Eq. (1):
+// One persistent, warp-specialised, single-pass kernel evaluates Eq. (1)
+// (P:76-78).  Per tile of m = 32*W*X elements:
 //   a1 load + fused FIR map (Eq. (2))
 //   a2 per-thread sequential chunk of X elements with zero state
 //      (the serial loop of P:206-214; work-efficient replacement of the
 //      element-level doubling of Phase 1)
 //   a3 warp carry propagation: Kogge-Stone over the 32 lanes with
-//      T(X*2^s), shuffles
-//   a4 block propagation of warp aggregates through shared memory
+//      T(X*2^s) and shuffles
+//   a4 block propagation of the warp aggregates through shared memory
+//
 //   a5 grid: decoupled look-back of the k carries with epoch-tagged status
-//      words (Phase 2; carry precomputation P:527-556;
-//      chunk ticket P:651-653; publish/wait P:668-683)
+//      words (Phase 2; carry precomputation P:527-556; chunk
+//      ticket P:651-653; publish / wait P:668-683)
 //   a6 carry-in distribution + correction y_u = l_u + sum_r S_r h^(r)_u
 //
 //   a7 store
-// Data movement: one producer warp issues TMA bulk copies
-// (cp.async.bulk, mbarrier complete_tx) of whole tiles into an S-stage
-// shared-memory ring and TMA bulk stores of the finished tiles; compute warps
-// only touch shared memory (odd X => conflict-free strided access).
+// Roles: warp W (producer) takes tickets and moves whole tiles with TMA bulk
+// copies (cp.async.bulk + mbarrier complete_tx) into an S-stage shared-memory
+// ring and back out with TMA bulk stores; warp W+1 (look-back) runs a5 for
+// the CTA's tiles in order; warps 0..W-1 (compute) run phase A (a1-a4) of
+// tile i+1 before phase B (a6-a7) of tile i, so the look-back latency of a
+// tile overlaps a whole tile of compute.
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
@@ -94,19 +98,16 @@ __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long lon
 // ------------------------------------------------------------- ring ops ----
 __device__ __forceinline__ uint32_t mad(uint32_t a, uint32_t b, uint32_t c) { return a * b + c; }
 __device__ __forceinline__ float mad(float a, float b, float c) { return __fmaf_rn(a, b, c); }
-__device__ __forceinline__ uint32_t bits(uint32_t v) { return v; }
-__device__ __forceinline__ uint32_t bits(float v) { return __float_as_uint(v); }
-template <typename T> __device__ __forceinline__ T from_bits(uint32_t b);
-template <> __device__ __forceinline__ uint32_t from_bits<uint32_t>(uint32_t b) { return b; }
-template <> __device__ __forceinline__ float from_bits<float>(uint32_t b) { return __uint_as_float(b); }
+__device__ __forceinline__ double mad(double a, double b, double c) { return __fma_rn(a, b, c); }
+
 
 // v[q] += sum_r Tm[q][r] * o[r]
-template <typename T, int K>
-__device__ __forceinline__ void matvec_acc(T (&v)[K], const T* Tm, const T (&o)[K]) {
-    T r_[K];
+template <typename A, int K>
+__device__ __forceinline__ void matvec_acc(A (&v)[K], const A* Tm, const A (&o)[K]) {
+    A r_[K];
 #pragma unroll
     for (int q = 0; q < K; q++) {
-        T acc = v[q];
+        A acc = v[q];
 #pragma unroll
         for (int r = 0; r < K; r++) acc = mad(Tm[q * kMaxK + r], o[r], acc);
         r_[q] = acc;
@@ -115,44 +116,114 @@ __device__ __forceinline__ void matvec_acc(T (&v)[K], const T* Tm, const T (&o)[
     for (int q = 0; q < K; q++) v[q] = r_[q];
 }
 
-// ------------------------------------------------------ the scan kernel ----
-template <int X, int W, int S>
-struct Smem {
-    static constexpr int M = 32 * W * X;
-    static constexpr int SW = M + kHalo;                       // words per stage
-    static constexpr size_t stage_bytes = (size_t)S * SW * 4;
-    static constexpr size_t bytes = stage_bytes + 2 * S * 8 /*bars*/ + S * 8 /*tile ids*/ +
-                                    (W * kMaxK + kMaxK) * 4 + 16;
+template <typename A>
+__device__ __forceinline__ A shfl_up(A v, int d) { return __shfl_up_sync(0xffffffffu, v, d); }
+template <typename A>
+__device__ __forceinline__ A shfl_down(A v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
+template <typename A>
+__device__ __forceinline__ A shfl_idx(A v, int l) { return __shfl_sync(0xffffffffu, v, l); }
+
+// ------------------------------------------------------ status words -------
+// Tile status: 2*kStatusWords 64-bit words per tile.  32-bit carries: word q
+// = {tag:32 | value:32} (one single-copy-atomic store each, so a reader
+// validates every component by its own tag).  fp64 carries: two words per
+// component, {tag | fp32 hi} and {tag | fp32 lo} with hi = fl(v),
+// lo = fl(v - hi) (a double-float split, ~48 significant bits).
+template <typename A> struct StatusIO;
+
+template <> struct StatusIO<uint32_t> {
+    static constexpr int kWords = 1;
+    __device__ static void pack(uint32_t v, uint32_t tag, unsigned long long* w) {
+        w[0] = ((unsigned long long)tag << 32) | v;
+    }
+    __device__ static bool unpack(const unsigned long long* w, uint32_t tag, uint32_t& v) {
+        v = (uint32_t)w[0];
+        return (uint32_t)(w[0] >> 32) == tag;
+    }
+};
+template <> struct StatusIO<float> {
+    static constexpr int kWords = 1;
+    __device__ static void pack(float v, uint32_t tag, unsigned long long* w) {
+        w[0] = ((unsigned long long)tag << 32) | __float_as_uint(v);
+    }
+    __device__ static bool unpack(const unsigned long long* w, uint32_t tag, float& v) {
+        v = __uint_as_float((uint32_t)w[0]);
+        return (uint32_t)(w[0] >> 32) == tag;
+    }
+};
+template <> struct StatusIO<double> {
+    static constexpr int kWords = 2;   // double-float split: hi = fl(v), lo = fl(v - hi)
+    __device__ static void pack(double v, uint32_t tag, unsigned long long* w) {
+        const float hi = __double2float_rn(v);
+        const float lo = __double2float_rn(v - (double)hi);
+        w[0] = ((unsigned long long)tag << 32) | __float_as_uint(hi);
+        w[1] = ((unsigned long long)tag << 32) | __float_as_uint(lo);
+    }
+    __device__ static bool unpack(const unsigned long long* w, uint32_t tag, double& v) {
+        v = (double)__uint_as_float((uint32_t)w[0]) + (double)__uint_as_float((uint32_t)w[1]);
+        return (uint32_t)(w[0] >> 32) == tag && (uint32_t)(w[1] >> 32) == tag;
+    }
 };
 
-template <typename T, int K, int P, int X, int W, int S, bool STORE>
-__global__ void __launch_bounds__((W + 1) * 32)
-plr_scan_kernel(const __grid_constant__ ScanParams<T> prm) {
-    using SM = Smem<X, W, S>;
-    constexpr int M = SM::M;
-    constexpr int SW = SM::SW;
-    constexpr int NC = W * 32;
+// ------------------------------------------------------ shared memory ------
+template <typename T, typename A, int K, int X, int W, int S>
+struct Layout {
+    static constexpr int M = 32 * W * X;
+    static constexpr int NC = 32 * W;
+    static constexpr int SW = M + kHalo;                        // words per stage
+    static constexpr size_t off_stage = 0;
+    static constexpr size_t off_E = (size_t)S * SW * sizeof(T);                       // [2][K][NC] A
+    static constexpr size_t off_Pw = off_E + 2 * (size_t)K * NC * sizeof(A);          // [2][W][K] A
+    static constexpr size_t off_At = off_Pw + 2 * (size_t)W * K * sizeof(A);          // [2][K] A
+    static constexpr size_t off_G = off_At + 2 * (size_t)kMaxK * sizeof(A);           // [2][K] A
+    static constexpr size_t off_wagg = off_G + 2 * (size_t)kMaxK * sizeof(A);         // [2][W][K] A
+    static constexpr size_t off_bar = (off_wagg + 2 * (size_t)W * kMaxK * sizeof(A) + 15) & ~(size_t)15;
+    // bars: full[S], done[S], agg[2], carry[2]
+    static constexpr size_t off_tile = off_bar + (2 * S + 4) * 8;                    // tile_of[S]
+    static constexpr size_t off_aggtile = off_tile + S * 8;                           // agg_tile[2]
+    static constexpr size_t bytes = off_aggtile + 2 * 8;
+};
+
+// ------------------------------------------------------ the scan kernel ----
+template <typename T, typename A, int K, int P, int X, int W, int S, bool STORE>
+__global__ void __launch_bounds__((W + 2) * 32)
+plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
+    using L = Layout<T, A, K, X, W, S>;
+    constexpr int M = L::M;
+    constexpr int SW = L::SW;
+    constexpr int NC = L::NC;
     constexpr int LOGW = (W >= 16) ? 4 : (W >= 8) ? 3 : (W >= 4) ? 2 : (W >= 2) ? 1 : 0;
     static_assert((1 << LOGW) == W, "W must be a power of two");
     static_assert(X >= K && X <= kMaxX && (X & 1), "X must be odd and >= K");
     static_assert(P <= kHalo, "halo");
+    using SIO = StatusIO<A>;
+    static_assert(K * SIO::kWords <= 2 * kStatusWords, "status words");
+    static_assert(S >= 3, "phase B of tile i runs after phase A of tile i+1: needs >= 3 stages");
 
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    T* stages = reinterpret_cast<T*>(smem_raw);
-    uint64_t* full_bar = reinterpret_cast<uint64_t*>(smem_raw + SM::stage_bytes);
+    extern __shared__ __align__(128) unsigned char smem[];
+    T* stages = reinterpret_cast<T*>(smem + L::off_stage);
+    A* sE = reinterpret_cast<A*>(smem + L::off_E);
+    A* sPw = reinterpret_cast<A*>(smem + L::off_Pw);
+    A* sAt = reinterpret_cast<A*>(smem + L::off_At);
+    A* sG = reinterpret_cast<A*>(smem + L::off_G);
+    A* wagg = reinterpret_cast<A*>(smem + L::off_wagg);
+    uint64_t* full_bar = reinterpret_cast<uint64_t*>(smem + L::off_bar);
     uint64_t* done_bar = full_bar + S;
-    long long* tile_of = reinterpret_cast<long long*>(done_bar + S);
-    T* wagg = reinterpret_cast<T*>(tile_of + S);               // [W][K]
-    T* bcast = wagg + W * kMaxK;                               // [K]
+    uint64_t* agg_bar = done_bar + S;
+    uint64_t* carry_bar = agg_bar + 2;
+    long long* tile_of = reinterpret_cast<long long*>(smem + L::off_tile);
+    long long* agg_tile = reinterpret_cast<long long*>(smem + L::off_aggtile);
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
     const long long ntiles = (long long)prm.ntiles;
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
+    const Tables<T, A>& tb = prm.tab;
 
     if (tid == 0) {
         for (int s = 0; s < S; s++) { mbar_init(&full_bar[s], 1); mbar_init(&done_bar[s], NC); }
+        for (int s = 0; s < 2; s++) { mbar_init(&agg_bar[s], 1); mbar_init(&carry_bar[s], 1); }
         fence_mbar_init();
     }
     __syncthreads();
@@ -166,7 +237,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T> prm) {
             const long long j = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
             tile_of[s] = j;
             if (j >= ntiles) { done = true; mbar_arrive(&full_bar[s]); return; }
-            if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_bar[s]); return; }   // consumers load it
+            if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_bar[s]); return; }   // compute loads it
             T* st = stages + (size_t)s * SW;
             if (j == 0) {
 #pragma unroll
@@ -200,23 +271,197 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T> prm) {
         return;
     }
 
+    // ===================================================== look-back warp ==
+    if (warp == W + 1) {
+        const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
+        constexpr int NW = K * SIO::kWords;
+        auto publish = [&](long long j, const A (&val)[K], uint32_t tag) {
+            unsigned long long* stj = prm.status + (size_t)j * (2 * kStatusWords);
+            unsigned long long w[NW];
+#pragma unroll
+            for (int q = 0; q < K; q++) SIO::pack(val[q], tag, &w[q * SIO::kWords]);
+#pragma unroll
+            for (int e = 0; e < NW; e++) if (lane == e) st_relaxed(stj + e, w[e]);
+        };
+        // read tile jj's K components; returns 2 inclusive, 1 aggregate, 0 not ready
+        auto read_status = [&](long long jj, A (&val)[K]) -> int {
+            const unsigned long long* sp = prm.status + (size_t)jj * (2 * kStatusWords);
+            unsigned long long w[NW];
+#pragma unroll
+            for (int e = 0; e < NW; e++) w[e] = ld_relaxed(sp + e);
+            bool allI = true, allA = true;
+#pragma unroll
+            for (int q = 0; q < K; q++) {
+                allI = SIO::unpack(&w[q * SIO::kWords], tagI, val[q]) && allI;
+                bool a2 = SIO::unpack(&w[q * SIO::kWords], tagA, val[q]);
+                allA = allA && a2;
+            }
+            return allI ? 2 : (allA ? 1 : 0);
+        };
+        for (int it = 0;; it++) {
+            const int slot = it & 1;
+            mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
+            const long long j = agg_tile[slot];
+            if (j >= ntiles) break;
+            A At[K];
+#pragma unroll
+            for (int q = 0; q < K; q++) At[q] = sAt[slot * kMaxK + q];
+            A Gp[K];
+            if (j == 0) {
+#pragma unroll
+                for (int q = 0; q < K; q++) Gp[q] = prm.y_hist != nullptr ? A(prm.y_hist[K - 1 - q]) : A(0);
+                A G[K];
+#pragma unroll
+                for (int q = 0; q < K; q++) G[q] = At[q];
+                matvec_acc<A, K>(G, tb.Tm, Gp);
+                publish(0, G, tagI);
+            } else if (prm.decay) {
+                // T(m) == 0: inclusive == aggregate; single-hop look-back
+                publish(j, At, tagI);
+                A v[K];
+                if (lane == 0) {
+                    while (read_status(j - 1, v) != 2) __nanosleep(32);
+                }
+#pragma unroll
+                for (int q = 0; q < K; q++) Gp[q] = shfl_idx(lane == 0 ? v[q] : A(0), 0);
+            } else {
+                publish(j, At, tagA);
+                A acc[K];
+                A Tacc[K * kMaxK];
+#pragma unroll
+                for (int q = 0; q < K; q++) {
+                    acc[q] = A(0);
+#pragma unroll
+                    for (int r = 0; r < kMaxK; r++) Tacc[q * kMaxK + r] = (q == r) ? A(1) : A(0);
+                }
+                long long base = j - 1;
+                int tpl = 1;                       // first window: 32 tiles, then 32*kTPL
+                int spins = 0;
+                for (;;) {
+                    // lane owns tiles base - lane*tpl - t, t < tpl (contiguous)
+                    A v[kTPL][K];
+                    int st[kTPL];
+                    int first_incl = kTPL;
+#pragma unroll
+                    for (int t = 0; t < kTPL; t++) {
+                        st[t] = 2;
+#pragma unroll
+                        for (int q = 0; q < K; q++) v[t][q] = A(0);
+                        if (t < tpl) {
+                            const long long jj = base - (long long)lane * tpl - t;
+                            if (jj >= 0) st[t] = read_status(jj, v[t]);
+                        }
+                    }
+#pragma unroll
+                    for (int t = kTPL - 1; t >= 0; t--)
+                        if (t < tpl && st[t] == 2) first_incl = t;
+                    bool ready = true;
+#pragma unroll
+                    for (int t = 0; t < kTPL; t++)
+                        if (t < tpl && t <= first_incl && st[t] == 0) ready = false;
+                    const unsigned incl = __ballot_sync(0xffffffffu, first_incl < tpl);
+                    const int dl = incl ? (__ffs(incl) - 1) : 32;
+                    const unsigned need = dl >= 31 ? 0xffffffffu : ((2u << dl) - 1u);
+                    const unsigned notready = __ballot_sync(0xffffffffu, !ready);
+                    if (notready & need) {                       // re-poll the window
+                        if (++spins > 2) __nanosleep(64);
+                        continue;
+                    }
+                    spins = 0;
+                    // per-lane Horner fold over its tiles (up to its first inclusive)
+                    const int last = (lane < dl) ? tpl - 1 : (lane == dl ? first_incl : -1);
+                    A r[K];
+#pragma unroll
+                    for (int q = 0; q < K; q++) r[q] = A(0);
+#pragma unroll
+                    for (int t = kTPL - 1; t >= 0; t--) {
+                        if (t <= last) {
+                            A nr[K];
+#pragma unroll
+                            for (int q = 0; q < K; q++) nr[q] = v[t][q];
+                            matvec_acc<A, K>(nr, tb.Tm, r);
+#pragma unroll
+                            for (int q = 0; q < K; q++) r[q] = nr[q];
+                        }
+                    }
+                    // tree over lanes: R = sum_l T(l * tpl * m) r_l
+                    const A* Tl5 = (tpl == 1) ? &tb.Tlb1[0][0] : &tb.Tlb8[0][0];
+#pragma unroll
+                    for (int s2 = 0; s2 < 5; s2++) {
+                        A o[K];
+#pragma unroll
+                        for (int q = 0; q < K; q++) o[q] = shfl_down(r[q], 1 << s2);
+                        matvec_acc<A, K>(r, Tl5 + s2 * kMaxK * kMaxK, o);
+                    }
+                    A R[K];
+#pragma unroll
+                    for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
+                    matvec_acc<A, K>(acc, Tacc, R);
+                    if (dl < 32) break;
+                    // next window, further back: Tacc *= T(32 * tpl * m)
+                    const A* Tw = (tpl == 1) ? tb.Tw1 : tb.Tw8;
+                    A nt[K * kMaxK];
+#pragma unroll
+                    for (int q = 0; q < K; q++)
+#pragma unroll
+                        for (int c2 = 0; c2 < K; c2++) {
+                            A a2 = A(0);
+#pragma unroll
+                            for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], Tw[t * kMaxK + c2], a2);
+                            nt[q * kMaxK + c2] = a2;
+                        }
+#pragma unroll
+                    for (int q = 0; q < K; q++)
+#pragma unroll
+                        for (int c2 = 0; c2 < K; c2++) Tacc[q * kMaxK + c2] = nt[q * kMaxK + c2];
+                    base -= 32LL * tpl;
+                    if (tpl == 1) {
+                        // the next window starts after this one; when it went
+                        // wide it covers 32*kTPL tiles per round trip
+                        tpl = kTPL;
+                        // Tacc currently maps the next (narrow-sized) step;
+                        // it already includes T(32 m), which is where the wide
+                        // window begins, so nothing else to adjust
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < K; q++) Gp[q] = acc[q];
+                A G[K];
+#pragma unroll
+                for (int q = 0; q < K; q++) G[q] = At[q];
+                matvec_acc<A, K>(G, tb.Tm, Gp);
+                publish(j, G, tagI);
+            }
+            if (lane == 0) {
+#pragma unroll
+                for (int q = 0; q < K; q++) sG[slot * kMaxK + q] = Gp[q];
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&carry_bar[slot]);
+        }
+        return;
+    }
+
     // ===================================================== compute warps ===
-    const Tables<T>& tb = prm.tab;
-    T Tl[K * K];                                                // T(X*lane)
+    A Tl[K * K];                                                // T(X*lane)
 #pragma unroll
     for (int e = 0; e < K * K; e++) Tl[e] = prm.lane_T[e * 32 + lane];
-    const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
 
-    for (int it = 0;; it++) {
+    // phase A of pipeline iteration `it`: returns the tile id (>= ntiles: stop)
+    auto phaseA = [&](int it) -> long long {
         const int s = it % S;
+        const int slot = it & 1;
         mbar_wait(&full_bar[s], (uint32_t)((it / S) & 1));
         const long long j = tile_of[s];
-        if (j >= ntiles) break;
+        if (j >= ntiles) {
+            if (tid == 0) { agg_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
+            return j;
+        }
         const bool ragged = (j == ntiles - 1) && last_ragged;
         T* st = stages + (size_t)s * SW;
-        const long long g0 = j * (long long)M + (long long)tid * X;   // global index of my first element
+        const long long g0 = j * (long long)M + (long long)tid * X;
 
-        // ---- a1: load my X elements (+ P halo) and apply the FIR map -----
+        // a1: my X elements (+ P halo), FIR map in the data type
         T xv[X + P];
         if (!ragged) {
             const T* base = st + kHalo + tid * X;
@@ -234,215 +479,115 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T> prm) {
                 xv[q] = v;
             }
         }
-        // ---- a2: sequential local recurrence with zero state --------------
-        T l[X];
+        // a2: sequential local recurrence with zero state, in A
+        A l[X];
 #pragma unroll
         for (int u = 0; u < X; u++) {
-            T acc = tb.alpha[0] * xv[P + u];
+            T t = tb.alpha[0] * xv[P + u];
 #pragma unroll
-            for (int q = 1; q <= P; q++) acc = mad(tb.alpha[q], xv[P + u - q], acc);
+            for (int q = 1; q <= P; q++) t = mad(tb.alpha[q], xv[P + u - q], t);
+            A acc = A(t);
 #pragma unroll
             for (int r = 1; r <= K; r++)
                 if (u - r >= 0) acc = mad(tb.c[r - 1], l[u - r], acc);
             l[u] = acc;
         }
-        // local carry A = (l_{X-1}, ..., l_{X-K})
-        T v[K];
+        A v[K];
 #pragma unroll
-        for (int q = 0; q < K; q++) v[q] = l[X - 1 - q];
+        for (int q = 0; q < K; q++) v[q] = l[X - 1 - q];       // local carry (l_{X-1}, ..., l_{X-K})
 
-        // ---- a3: warp inclusive scan with T(X * 2^s) ----------------------
+        // a3: warp inclusive scan with T(X * 2^s)
 #pragma unroll
         for (int s2 = 0; s2 < 5; s2++) {
-            T o[K];
+            A o[K];
 #pragma unroll
-            for (int q = 0; q < K; q++) o[q] = __shfl_up_sync(0xffffffffu, v[q], 1 << s2);
-            if (lane >= (1 << s2)) matvec_acc<T, K>(v, tb.Twarp[s2], o);
+            for (int q = 0; q < K; q++) o[q] = shfl_up(v[q], 1 << s2);
+            if (lane >= (1 << s2)) matvec_acc<A, K>(v, tb.Twarp[s2], o);
         }
-        T E[K];                                                  // warp-exclusive prefix
 #pragma unroll
         for (int q = 0; q < K; q++) {
-            T t = __shfl_up_sync(0xffffffffu, v[q], 1);
-            E[q] = lane == 0 ? T(0) : t;
+            const A e = shfl_up(v[q], 1);
+            sE[(slot * K + q) * NC + tid] = lane == 0 ? A(0) : e;  // warp-exclusive prefix
         }
         if (lane == 31) {
 #pragma unroll
-            for (int q = 0; q < K; q++) wagg[warp * kMaxK + q] = v[q];
+            for (int q = 0; q < K; q++) wagg[(slot * W + warp) * kMaxK + q] = v[q];
         }
-        named_sync(1, NC);
+        named_sync(1, NC);                                      // all x reads and wagg writes done
 
-        // ---- a4: scan of the W warp aggregates with T(32X * 2^s) ----------
-        T u_[K];
+        // keep the chunk values for phase B in place of x (data type)
 #pragma unroll
-        for (int q = 0; q < K; q++) u_[q] = lane < W ? wagg[lane * kMaxK + q] : T(0);
+        for (int u = 0; u < X; u++) st[kHalo + tid * X + u] = T(l[u]);
+
+        // a4: scan of the W warp aggregates with T(32X * 2^s)
+        A u_[K];
+#pragma unroll
+        for (int q = 0; q < K; q++) u_[q] = lane < W ? wagg[(slot * W + lane) * kMaxK + q] : A(0);
 #pragma unroll
         for (int s2 = 0; s2 < LOGW; s2++) {
-            T o[K];
+            A o[K];
 #pragma unroll
-            for (int q = 0; q < K; q++) o[q] = __shfl_up_sync(0xffffffffu, u_[q], 1 << s2);
-            if (lane >= (1 << s2)) matvec_acc<T, K>(u_, tb.Tblk[s2], o);
+            for (int q = 0; q < K; q++) o[q] = shfl_up(u_[q], 1 << s2);
+            if (lane >= (1 << s2)) matvec_acc<A, K>(u_, tb.Tblk[s2], o);
         }
-        T Pw[K], At[K];
 #pragma unroll
         for (int q = 0; q < K; q++) {
-            T t = __shfl_sync(0xffffffffu, u_[q], (warp + 31) & 31);
-            Pw[q] = warp == 0 ? T(0) : t;
-            At[q] = __shfl_sync(0xffffffffu, u_[q], W - 1);     // tile aggregate
+            const A pw = shfl_idx(u_[q], (warp + 31) & 31);
+            const A at = shfl_idx(u_[q], W - 1);                // tile aggregate
+            if (lane == 0) sPw[(slot * W + warp) * K + q] = warp == 0 ? A(0) : pw;
+            if (tid == 0) sAt[slot * kMaxK + q] = at;
         }
+        // wagg is double-buffered by slot: its next writer (tile it+2) runs
+        // after every warp passed tile it+1's barrier
+        __syncwarp();                                           // sPw (lane 0) visible to the warp
+        if (tid == 0) { agg_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
+        return j;
+    };
 
-        // ---- a5: decoupled look-back (warp 0) -----------------------------
-        if (warp == 0) {
-            T Gp[K];
-            unsigned long long* stj = prm.status + (size_t)j * kStatusWords;
-            auto publish = [&](const T (&val)[K], uint32_t tag) {
-                T mine = T(0);
+    // phase B of pipeline iteration `it` (tile id j)
+    auto phaseB = [&](int it, long long j) {
+        const int s = it % S;
+        const int slot = it & 1;
+        mbar_wait(&carry_bar[slot], (uint32_t)((it >> 1) & 1));
+        const bool ragged = (j == ntiles - 1) && last_ragged;
+        T* st = stages + (size_t)s * SW;
+        const long long g0 = j * (long long)M + (long long)tid * X;
+        A Gp[K], Win[K], Sst[K];
 #pragma unroll
-                for (int q = 0; q < K; q++) if (lane == q) mine = val[q];
-                if (lane < K) st_relaxed(stj + lane, ((unsigned long long)tag << 32) | bits(mine));
-            };
-            if (j == 0) {
-#pragma unroll
-                for (int q = 0; q < K; q++) Gp[q] = prm.y_hist != nullptr ? prm.y_hist[K - 1 - q] : T(0);
-                T G[K];
-#pragma unroll
-                for (int q = 0; q < K; q++) G[q] = At[q];
-                matvec_acc<T, K>(G, tb.Tlb[0], Gp);
-                publish(G, tagI);
-            } else if (prm.decay) {
-                // T(m) == 0: the inclusive carry equals the aggregate, publish
-                // it at once; the look-back is a single hop.
-                publish(At, tagI);
-                const unsigned long long* sp = prm.status + (size_t)(j - 1) * kStatusWords;
-                uint32_t word = 0;
-                if (lane < K) {
-                    unsigned long long w;
-                    do { w = ld_relaxed(sp + lane); } while ((uint32_t)(w >> 32) != tagI);
-                    word = (uint32_t)w;
-                }
-#pragma unroll
-                for (int q = 0; q < K; q++) Gp[q] = from_bits<T>(__shfl_sync(0xffffffffu, word, q));
-            } else {
-                publish(At, tagA);
-                T acc[K];
-                T Tacc[K * kMaxK];
-#pragma unroll
-                for (int q = 0; q < K; q++) {
-                    acc[q] = T(0);
-#pragma unroll
-                    for (int r = 0; r < kMaxK; r++) Tacc[q * kMaxK + r] = (q == r) ? T(1) : T(0);
-                }
-                long long base = j - 1;
-                for (;;) {
-                    const long long jj = base - lane;
-                    int stt = 2;                                   // jj < 0: never needed
-                    T val[K];
-#pragma unroll
-                    for (int q = 0; q < K; q++) val[q] = T(0);
-                    if (jj >= 0) {
-                        const unsigned long long* sp = prm.status + (size_t)jj * kStatusWords;
-                        unsigned long long w[K];
-#pragma unroll
-                        for (int q = 0; q < K; q++) w[q] = ld_relaxed(sp + q);
-                        bool allI = true, allA = true;
-#pragma unroll
-                        for (int q = 0; q < K; q++) {
-                            const uint32_t tg = (uint32_t)(w[q] >> 32);
-                            allI = allI && tg == tagI;
-                            allA = allA && tg == tagA;
-                            val[q] = from_bits<T>((uint32_t)w[q]);
-                        }
-                        stt = allI ? 2 : (allA ? 1 : 0);
-                    }
-                    const unsigned incl = __ballot_sync(0xffffffffu, stt == 2);
-                    const int d = incl ? (__ffs(incl) - 1) : 32;
-                    const unsigned need = d >= 31 ? 0xffffffffu : ((2u << d) - 1u);
-                    const unsigned notready = __ballot_sync(0xffffffffu, stt == 0);
-                    if (notready & need) continue;                 // re-poll the window
-                    if (lane > d) {
-#pragma unroll
-                        for (int q = 0; q < K; q++) val[q] = T(0);
-                    }
-                    // fold: R = sum_{l<=d} T(l*m) val_l  (tree over lanes)
-#pragma unroll
-                    for (int s2 = 0; s2 < 5; s2++) {
-                        T o[K];
-#pragma unroll
-                        for (int q = 0; q < K; q++) o[q] = __shfl_down_sync(0xffffffffu, val[q], 1 << s2);
-                        matvec_acc<T, K>(val, tb.Tlb[s2], o);
-                    }
-                    T R[K];
-#pragma unroll
-                    for (int q = 0; q < K; q++) R[q] = __shfl_sync(0xffffffffu, val[q], 0);
-                    matvec_acc<T, K>(acc, Tacc, R);
-                    if (d < 32) break;
-                    // the next window is 32 tiles further back: Tacc *= T(32m)
-                    T nt[K * kMaxK];
-#pragma unroll
-                    for (int q = 0; q < K; q++)
-#pragma unroll
-                        for (int r = 0; r < K; r++) {
-                            T a2 = T(0);
-#pragma unroll
-                            for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], tb.Tlb[5][t * kMaxK + r], a2);
-                            nt[q * kMaxK + r] = a2;
-                        }
-#pragma unroll
-                    for (int e = 0; e < K * kMaxK; e++) Tacc[e] = nt[e];
-                    base -= 32;
-                }
-#pragma unroll
-                for (int q = 0; q < K; q++) Gp[q] = acc[q];
-                T G[K];
-#pragma unroll
-                for (int q = 0; q < K; q++) G[q] = At[q];
-                matvec_acc<T, K>(G, tb.Tlb[0], Gp);
-                publish(G, tagI);
-            }
-            if (lane < K) {
-                T mine = T(0);
-#pragma unroll
-                for (int q = 0; q < K; q++) if (lane == q) mine = Gp[q];
-                bcast[lane] = mine;
-            }
+        for (int q = 0; q < K; q++) {
+            Gp[q] = sG[slot * kMaxK + q];
+            Win[q] = sPw[(slot * W + warp) * K + q];
         }
-        named_sync(1, NC);
-
-        // ---- a6: carry-in and correction ----------------------------------
-        T Gp[K];
-#pragma unroll
-        for (int q = 0; q < K; q++) Gp[q] = bcast[q];
-        T Win[K];
-#pragma unroll
-        for (int q = 0; q < K; q++) Win[q] = Pw[q];
-        matvec_acc<T, K>(Win, tb.Twin[warp], Gp);              // warp carry-in
-        T Sst[K];
+        matvec_acc<A, K>(Win, tb.Twin[warp], Gp);              // warp carry-in
 #pragma unroll
         for (int q = 0; q < K; q++) {                           // thread carry-in
-            T acc = E[q];
+            A acc = sE[(slot * K + q) * NC + tid];
 #pragma unroll
             for (int r = 0; r < K; r++) acc = mad(Tl[q * K + r], Win[r], acc);
             Sst[q] = acc;
         }
+        T Sd[K];
+#pragma unroll
+        for (int q = 0; q < K; q++) Sd[q] = T(Sst[q]);
+        T* base = st + kHalo + tid * X;
+        T yv[X];
 #pragma unroll
         for (int u = 0; u < X; u++) {
-            T acc = l[u];
+            T acc = base[u];
 #pragma unroll
-            for (int r = 0; r < K; r++) acc = mad(tb.H[u][r], Sst[r], acc);
-            l[u] = acc;
+            for (int r = 0; r < K; r++) acc = mad(tb.H[u][r], Sd[r], acc);
+            yv[u] = acc;
         }
-
-        // ---- a7: write back ----------------------------------------------
         if (!ragged) {
             if (STORE) {
-                T* base = st + kHalo + tid * X;
 #pragma unroll
-                for (int u = 0; u < X; u++) base[u] = l[u];
+                for (int u = 0; u < X; u++) base[u] = yv[u];
             }
         } else if (STORE) {
 #pragma unroll
             for (int u = 0; u < X; u++) {
                 const long long i = g0 + u;
-                if ((unsigned long long)i < n) prm.y[i] = l[u];
+                if ((unsigned long long)i < n) prm.y[i] = yv[u];
             }
         }
         if (prm.y_tail != nullptr) {
@@ -451,12 +596,21 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T> prm) {
 #pragma unroll
                 for (int u = 0; u < X; u++) {
                     const long long i = g0 + u;
-                    if (i >= lo && i < (long long)n) prm.y_tail[i - lo] = l[u];
+                    if (i >= lo && i < (long long)n) prm.y_tail[i - lo] = yv[u];
                 }
             }
         }
         fence_proxy_async();
         mbar_arrive(&done_bar[s]);
+    };
+
+    long long jprev = phaseA(0);
+    if (jprev >= ntiles) return;
+    for (int it = 1;; it++) {
+        const long long j = phaseA(it);
+        phaseB(it - 1, jprev);
+        if (j >= ntiles) break;
+        jprev = j;
     }
 }
 

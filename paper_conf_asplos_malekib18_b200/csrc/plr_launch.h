@@ -33,10 +33,9 @@ Geometry default_geometry(plr_dtype dtype, int k, int p);
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm);
 
-// per-dtype entry points
-cudaError_t launch_scan_i32(const PlanTables& pt, const LaunchArgs& la);
-cudaError_t launch_scan_f32(const PlanTables& pt, const LaunchArgs& la);
-cudaError_t occupancy_i32(const PlanTables& pt, int* ctas_per_sm);
-cudaError_t occupancy_f32(const PlanTables& pt, int* ctas_per_sm);
+// per-(data, accumulation) type entry points (plr_scan_*.cu)
+cudaError_t launch_scan_i32(const Tables<uint32_t, uint32_t>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_scan_f32(const Tables<float, float>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_scan_f64acc(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
 
 }  // namespace plr

@@ -82,21 +82,27 @@ void store_mat(const Mat<R>& m, T* dst, Cvt cvt) {
             dst[q * kMaxK + r] = (q < m.k && r < m.k) ? cvt(m.at(q, r)) : T(0);
 }
 
-template <typename R, typename T, typename Cvt>
-void fill_tables(const Mat<R>& M, int k, Geometry geo, Tables<T>* tb, T* lane, Cvt cvt) {
+// Fill every transfer-matrix table of Tables<T, A>; cvtA converts the ring
+// value to the accumulation type, cvtT to the data type (per-element H).
+template <typename R, typename T, typename A, typename CvtT, typename CvtA>
+void fill_tables(const Mat<R>& M, int k, Geometry geo, Tables<T, A>* tb, A* lane, CvtT cvtT, CvtA cvtA) {
     const uint64_t X = geo.X, m = (uint64_t)geo.tile();
     for (int u = 0; u < kMaxX; u++) {
         Mat<R> Tu = mpow(M, (uint64_t)u + 1);
-        for (int r = 0; r < kMaxK; r++) tb->H[u][r] = (u < geo.X && r < k) ? cvt(Tu.at(0, r)) : T(0);
+        for (int r = 0; r < kMaxK; r++) tb->H[u][r] = (u < geo.X && r < k) ? cvtT(Tu.at(0, r)) : T(0);
     }
-    for (int s = 0; s < 5; s++) store_mat(mpow(M, X << s), tb->Twarp[s], cvt);
-    for (int s = 0; s < 4; s++) store_mat(mpow(M, (32 * X) << s), tb->Tblk[s], cvt);
-    for (int w = 0; w < kMaxW; w++) store_mat(mpow(M, 32 * X * (uint64_t)w), tb->Twin[w], cvt);
-    for (int s = 0; s < 6; s++) store_mat(mpow(M, m << s), tb->Tlb[s], cvt);
+    for (int s = 0; s < 5; s++) store_mat(mpow(M, X << s), tb->Twarp[s], cvtA);
+    for (int s = 0; s < 4; s++) store_mat(mpow(M, (32 * X) << s), tb->Tblk[s], cvtA);
+    for (int w = 0; w < kMaxW; w++) store_mat(mpow(M, 32 * X * (uint64_t)w), tb->Twin[w], cvtA);
+    store_mat(mpow(M, m), tb->Tm, cvtA);
+    for (int s = 0; s < 5; s++) store_mat(mpow(M, m << s), tb->Tlb1[s], cvtA);
+    for (int s = 0; s < 5; s++) store_mat(mpow(M, (kTPL * m) << s), tb->Tlb8[s], cvtA);
+    store_mat(mpow(M, 32 * m), tb->Tw1, cvtA);
+    store_mat(mpow(M, 32 * kTPL * m), tb->Tw8, cvtA);
     for (int l = 0; l < 32; l++) {
         Mat<R> Tl = mpow(M, X * (uint64_t)l);
         for (int q = 0; q < k; q++)
-            for (int r = 0; r < k; r++) lane[(q * k + r) * 32 + l] = cvt(Tl.at(q, r));
+            for (int r = 0; r < k; r++) lane[(q * k + r) * 32 + l] = cvtA(Tl.at(q, r));
     }
 }
 
@@ -144,7 +150,8 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         for (int j = 0; j <= kMaxP; j++) pt.ti.alpha[j] = j <= p ? pt.a_u[j] : 0u;
         for (int j = 0; j < kMaxK; j++) pt.ti.c[j] = j < k ? c[j] : 0u;
         Mat<uint32_t> M = companion<uint32_t>(c, k);
-        fill_tables(M, k, geo, &pt.ti, pt.lane_i, [](uint32_t v) { return v; });
+        auto id = [](uint32_t v) { return v; };
+        fill_tables(M, k, geo, &pt.ti, pt.lane_i, id, id);
         // class: all factors 1 -> ONES; single unit feedback
         // coefficient -> PERM (0/1 repeating factors); otherwise POLY
         int nnz = 0, ones = 0;
@@ -157,10 +164,16 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         double c[kMaxK] = {0}, al[kMaxP + 1] = {0};
         for (int j = 0; j <= p; j++) al[j] = pt.a_d[j] = (double)(float)a[j];
         for (int j = 0; j < k; j++) c[j] = pt.b_d[j] = (double)(float)b[j];
-        for (int j = 0; j <= kMaxP; j++) pt.tf.alpha[j] = j <= p ? (float)al[j] : 0.0f;
+        for (int j = 0; j <= kMaxP; j++) pt.tf.alpha[j] = pt.td.alpha[j] = j <= p ? (float)al[j] : 0.0f;
         for (int j = 0; j < kMaxK; j++) pt.tf.c[j] = j < k ? (float)c[j] : 0.0f;
+        for (int j = 0; j < kMaxK; j++) pt.td.c[j] = j < k ? c[j] : 0.0;
         Mat<double> M = companion<double>(c, k);
-        fill_tables(M, k, geo, &pt.tf, pt.lane_f, [](double v) { return ftz(v); });
+        auto f32 = [](double v) { return ftz(v); };
+        // fp64 accumulation keeps denormal-range values that fp32 would flush;
+        // flush them too so both precisions see the same (exactly 0) tails
+        auto f64 = [](double v) { return std::fabs(v) < (double)FLT_MIN ? 0.0 : v; };
+        fill_tables(M, k, geo, &pt.tf, pt.lane_f, f32, f32);
+        fill_tables(M, k, geo, &pt.td, pt.lane_d, f32, f64);
         // DECAY: the fp32 impulse response g of (1: c) becomes
         // exactly 0 and stays 0.  g_0 = 1, g_u = sum_j c_j g_{u-j}.
         const int64_t cap = 1 << 16;
@@ -174,9 +187,21 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         }
         const bool decays = last < cap / 2;
         bool tm_zero = true;
-        for (int e = 0; e < kMaxK * kMaxK; e++) tm_zero = tm_zero && pt.tf.Tlb[0][e] == 0.0f;
+        for (int e = 0; e < kMaxK * kMaxK; e++) tm_zero = tm_zero && pt.tf.Tm[e] == 0.0f && pt.td.Tm[e] == 0.0;
         pt.decay_flag = (decays && tm_zero) ? 1 : 0;
         pt.cls = decays ? PLR_CLASS_DECAY : PLR_CLASS_FLOAT;
+        // Accumulation precision (reading R16).  The zero-state
+        // chunk values l_u and the carries reach ~sum|a| * sum|g| while the
+        // outputs stay small, and their rounding errors are amplified by the
+        // correction factors again (~sum|g|): a-priori bound
+        // eps32 * sum|a| * (sum|g|)^2.  Above 1e-3 (10x the 1e-4 tolerance)
+        // accumulate the recurrence and every carry in fp64 (B200 fp64 runs at
+        // half the fp32 rate); data, FIR and the final correction stay fp32.
+        double sa = 0.0, sg = 0.0;
+        for (int j = 0; j <= p; j++) sa += std::fabs(al[j]);
+        for (int64_t u = 0; u < cap; u++) sg += std::fabs(g[u]);
+        pt.cond_bound = std::ldexp(1.0, -24) * sa * sg * sg;
+        pt.acc64 = (!decays || !(pt.cond_bound <= 1e-3)) ? 1 : 0;
         if (decays) {
             pt.decay_len = last;
             // free response of the augmented state (x_{-4..-1}, y_{-4..-1})
