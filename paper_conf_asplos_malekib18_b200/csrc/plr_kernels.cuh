@@ -165,6 +165,42 @@ template <> struct StatusIO<double> {
     }
 };
 
+// publish carry vector `val` of tile j with `tag`; lanes 0..K*kWords-1 of the
+// calling warp each store one 64-bit word
+template <typename A, int K>
+__device__ __forceinline__ void publish_status(unsigned long long* status, long long j, const A (&val)[K],
+                                               uint32_t tag, int lane) {
+    using SIO = StatusIO<A>;
+    constexpr int NW = K * SIO::kWords;
+    unsigned long long* stj = status + (size_t)j * (2 * kStatusWords);
+    unsigned long long w[NW];
+#pragma unroll
+    for (int q = 0; q < K; q++) SIO::pack(val[q], tag, &w[q * SIO::kWords]);
+#pragma unroll
+    for (int e = 0; e < NW; e++) if (lane == e) st_relaxed(stj + e, w[e]);
+}
+
+// read tile jj's K components: 2 inclusive, 1 aggregate, 0 not ready
+template <typename A, int K>
+__device__ __forceinline__ int read_status(const unsigned long long* status, long long jj, A (&val)[K],
+                                           uint32_t tagA, uint32_t tagI) {
+    using SIO = StatusIO<A>;
+    constexpr int NW = K * SIO::kWords;
+    const unsigned long long* sp = status + (size_t)jj * (2 * kStatusWords);
+    unsigned long long w[NW];
+#pragma unroll
+    for (int e = 0; e < NW; e++) w[e] = ld_relaxed(sp + e);
+    bool allI = true, allA = true;
+#pragma unroll
+    for (int q = 0; q < K; q++) {
+        const bool i1 = SIO::unpack(&w[q * SIO::kWords], tagI, val[q]);
+        const bool a1 = SIO::unpack(&w[q * SIO::kWords], tagA, val[q]);
+        allI = allI && i1;
+        allA = allA && a1;
+    }
+    return allI ? 2 : (allA ? 1 : 0);
+}
+
 // ------------------------------------------------------ shared memory ------
 template <typename T, typename A, int K, int X, int W, int S>
 struct Layout {
@@ -272,60 +308,31 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     }
 
     // ===================================================== look-back warp ==
+    // Runs a5 for the CTA's tiles in ticket order.  It learns the tile id from
+    // the full barrier (as soon as the tile is loaded) and walks back without
+    // waiting for the tile's own aggregate, which the compute warps publish.
     if (warp == W + 1) {
         const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
-        constexpr int NW = K * SIO::kWords;
-        auto publish = [&](long long j, const A (&val)[K], uint32_t tag) {
-            unsigned long long* stj = prm.status + (size_t)j * (2 * kStatusWords);
-            unsigned long long w[NW];
-#pragma unroll
-            for (int q = 0; q < K; q++) SIO::pack(val[q], tag, &w[q * SIO::kWords]);
-#pragma unroll
-            for (int e = 0; e < NW; e++) if (lane == e) st_relaxed(stj + e, w[e]);
-        };
-        // read tile jj's K components; returns 2 inclusive, 1 aggregate, 0 not ready
-        auto read_status = [&](long long jj, A (&val)[K]) -> int {
-            const unsigned long long* sp = prm.status + (size_t)jj * (2 * kStatusWords);
-            unsigned long long w[NW];
-#pragma unroll
-            for (int e = 0; e < NW; e++) w[e] = ld_relaxed(sp + e);
-            bool allI = true, allA = true;
-#pragma unroll
-            for (int q = 0; q < K; q++) {
-                allI = SIO::unpack(&w[q * SIO::kWords], tagI, val[q]) && allI;
-                bool a2 = SIO::unpack(&w[q * SIO::kWords], tagA, val[q]);
-                allA = allA && a2;
-            }
-            return allI ? 2 : (allA ? 1 : 0);
-        };
         for (int it = 0;; it++) {
+            const int s = it % S;
             const int slot = it & 1;
-            mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
-            const long long j = agg_tile[slot];
+            mbar_wait(&full_bar[s], (uint32_t)((it / S) & 1));
+            const long long j = tile_of[s];
             if (j >= ntiles) break;
-            A At[K];
-#pragma unroll
-            for (int q = 0; q < K; q++) At[q] = sAt[slot * kMaxK + q];
-            A Gp[K];
+            A Gp[K];                                           // G_{j-1}: carries entering tile j
             if (j == 0) {
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = prm.y_hist != nullptr ? A(prm.y_hist[K - 1 - q]) : A(0);
-                A G[K];
-#pragma unroll
-                for (int q = 0; q < K; q++) G[q] = At[q];
-                matvec_acc<A, K>(G, tb.Tm, Gp);
-                publish(0, G, tagI);
             } else if (prm.decay) {
-                // T(m) == 0: inclusive == aggregate; single-hop look-back
-                publish(j, At, tagI);
+                // T(m) == 0: every tile published inclusive == aggregate at
+                // once; the look-back is a single hop
                 A v[K];
                 if (lane == 0) {
-                    while (read_status(j - 1, v) != 2) __nanosleep(32);
+                    while (read_status<A, K>(prm.status, j - 1, v, tagA, tagI) != 2) __nanosleep(20);
                 }
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = shfl_idx(lane == 0 ? v[q] : A(0), 0);
             } else {
-                publish(j, At, tagA);
                 A acc[K];
                 A Tacc[K * kMaxK];
 #pragma unroll
@@ -349,7 +356,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                         for (int q = 0; q < K; q++) v[t][q] = A(0);
                         if (t < tpl) {
                             const long long jj = base - (long long)lane * tpl - t;
-                            if (jj >= 0) st[t] = read_status(jj, v[t]);
+                            if (jj >= 0) st[t] = read_status<A, K>(prm.status, jj, v[t], tagA, tagI);
                         }
                     }
 #pragma unroll
@@ -364,7 +371,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     const unsigned need = dl >= 31 ? 0xffffffffu : ((2u << dl) - 1u);
                     const unsigned notready = __ballot_sync(0xffffffffu, !ready);
                     if (notready & need) {                       // re-poll the window
-                        if (++spins > 2) __nanosleep(64);
+                        if (++spins > 4) __nanosleep(32);
                         continue;
                     }
                     spins = 0;
@@ -398,7 +405,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
                     matvec_acc<A, K>(acc, Tacc, R);
                     if (dl < 32) break;
-                    // next window, further back: Tacc *= T(32 * tpl * m)
+                    // the next window lies 32*tpl tiles further back: Tacc *= T(32 tpl m)
                     const A* Tw = (tpl == 1) ? tb.Tw1 : tb.Tw8;
                     A nt[K * kMaxK];
 #pragma unroll
@@ -415,29 +422,29 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
                         for (int c2 = 0; c2 < K; c2++) Tacc[q * kMaxK + c2] = nt[q * kMaxK + c2];
                     base -= 32LL * tpl;
-                    if (tpl == 1) {
-                        // the next window starts after this one; when it went
-                        // wide it covers 32*kTPL tiles per round trip
-                        tpl = kTPL;
-                        // Tacc currently maps the next (narrow-sized) step;
-                        // it already includes T(32 m), which is where the wide
-                        // window begins, so nothing else to adjust
-                    }
+                    tpl = kTPL;
                 }
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = acc[q];
-                A G[K];
-#pragma unroll
-                for (int q = 0; q < K; q++) G[q] = At[q];
-                matvec_acc<A, K>(G, tb.Tm, Gp);
-                publish(j, G, tagI);
             }
+            // the tile's own aggregate (phase A) is needed for its inclusive carry
+            mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
             if (lane == 0) {
 #pragma unroll
                 for (int q = 0; q < K; q++) sG[slot * kMaxK + q] = Gp[q];
             }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&carry_bar[slot]);
+            if (!prm.decay || j == 0) {
+                A G[K];
+#pragma unroll
+                for (int q = 0; q < K; q++) G[q] = sAt[slot * kMaxK + q];
+                matvec_acc<A, K>(G, tb.Tm, Gp);                // G_j = A_j + T(m) G_{j-1}
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&carry_bar[slot]);
+                publish_status<A, K>(prm.status, j, G, tagI, lane);
+            } else {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&carry_bar[slot]);
+            }
         }
         return;
     }
@@ -536,6 +543,14 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             const A at = shfl_idx(u_[q], W - 1);                // tile aggregate
             if (lane == 0) sPw[(slot * W + warp) * K + q] = warp == 0 ? A(0) : pw;
             if (tid == 0) sAt[slot * kMaxK + q] = at;
+        }
+        // publish the tile aggregate at once: "P" for the generic
+        // look-back; for DECAY the inclusive carry equals the aggregate
+        if (warp == 0 && (j > 0 || prm.decay)) {
+            A At[K];
+#pragma unroll
+            for (int q = 0; q < K; q++) At[q] = shfl_idx(u_[q], W - 1);
+            publish_status<A, K>(prm.status, j, At, prm.decay ? 2u * prm.epoch + 1u : 2u * prm.epoch, lane);
         }
         // wagg is double-buffered by slot: its next writer (tile it+2) runs
         // after every warp passed tile it+1's barrier

@@ -104,9 +104,12 @@ def structured_input(kind: str, n: int, dtype: str) -> np.ndarray:
         if n:
             x[0] = 1
         return x
-    if kind == "alternating":          # the worked example's input pattern
+    if kind == "alternating":
         i = np.arange(n, dtype=np.int64)
-        v = np.where(i % 2 == 0, 1, -1) * (i + 3)
+        if dtype == "int32":           # the worked example's input pattern
+            v = np.where(i % 2 == 0, 1, -1) * (i + 3)
+        else:                          # unit amplitude: float workloads live in [-1, 1)
+            v = np.where(i % 2 == 0, 1.0, -1.0)
         return v.astype(npdt)
     if kind == "extremes":
         v = np.array([2 ** 31 - 1, -(2 ** 31), -1, 1], dtype=np.int64)
