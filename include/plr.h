@@ -114,6 +114,12 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info);
  * for PLR_FLOAT32 (rounded from fp64, denormals flushed).  Host memory. */
 plr_status plr_plan_factor_lists(const plr_plan* plan, int64_t m, void* out);
 
+/* Debug counters of the generic look-back, enabled by PLR_STATS=1 in the
+ * environment at plan creation (otherwise all zero): out[0] look-backs,
+ * out[1] windows read, out[2] waits on a not-ready tile, out[3] summed
+ * depth in tiles.  Synchronous; reset != 0 clears them.  Host memory. */
+plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out /* 8 */, int reset);
+
 /* y[0..n) = recurrence over x[0..n) with zero initial conditions.
  * x, y: device pointers of the plan's dtype. */
 plr_status plr_execute(plr_plan* plan, const void* x, void* y, size_t n, void* stream);

@@ -25,6 +25,7 @@ _SIGS = {
     "plr_plan_destroy": ([_P], _st),
     "plr_plan_get_info": ([_P, _P], _st),
     "plr_plan_factor_lists": ([_P, ctypes.c_int64, _P], _st),
+    "plr_plan_debug_stats": ([_P, _P, _I], _st),
     "plr_execute": ([_P, _P, _P, _S, _P], _st),
     "plr_execute_continue": ([_P, _P, _P, _S, _P, _P, _P], _st),
     "plr_reduce": ([_P, _P, _S, _P, _P], _st),
@@ -147,6 +148,12 @@ class Plan:
         d["dtype"] = "int32" if d["dtype"] == 0 else "float32"
         return d
 
+    def debug_stats(self, reset: bool = False) -> dict:
+        """Look-back counters (plan created with PLR_STATS=1 in the environment)."""
+        buf = (ctypes.c_uint64 * 8)()
+        _check(lib.plr_plan_debug_stats(self._h, buf, int(reset)), "plr_plan_debug_stats")
+        return {"lookbacks": buf[0], "windows": buf[1], "waits": buf[2], "depth_sum": buf[3]}
+
     def factor_lists(self, m: int):
         """The k seed-extended correction-factor lists (Sec. 2.1) as planned."""
         import numpy as np
@@ -200,8 +207,9 @@ class Plan:
     def combine(self, payloads, rank: int, world: int, hist=None, stream=None):
         """Boundary history of `rank` from all ranks' payloads (device)."""
         torch = _torch()
-        if hist is None:
-            hist = torch.zeros(8, dtype=torch.int32, device=payloads.device)
+        if hist is None:                        # 8 slots x_{-4..-1}, y_{-4..-1} in the plan's dtype
+            hist = torch.zeros(8, dtype=torch.int32 if self.dtype == "int32" else torch.float32,
+                               device=payloads.device)
         _check(lib.plr_combine(self._h, ctypes.c_void_p(payloads.data_ptr()), rank, world,
                                ctypes.c_void_p(hist.data_ptr()), _stream_ptr(stream)), "plr_combine")
         return hist

@@ -46,6 +46,7 @@ struct plr_plan {
     void* d_lane = nullptr;
     float* d_fix = nullptr;
     bool dirty = false;
+    unsigned long long* d_stats = nullptr;   // look-back counters when PLR_STATS=1
     // sharded path scratch
     unsigned char* d_send = nullptr;
     unsigned char* d_recv = nullptr;
@@ -229,6 +230,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.decay = plan->pt.decay_flag;
     la.x_hist = x_hist; la.y_hist = y_hist; la.y_tail = y_tail;
     la.lane_T = plan->d_lane;
+    la.stats = plan->d_stats;
     la.grid = (int)grid;
     la.store = store;
     la.stream = stream;
@@ -287,6 +289,7 @@ plr_status plr_plan_destroy(plr_plan* plan) {
     cudaFree(plan->d_send);
     cudaFree(plan->d_recv);
     cudaFree(plan->d_hist);
+    cudaFree(plan->d_stats);
     for (int i = 0; i < 3; i++) {
         cudaFree(plan->h_dx[i]);
         cudaFree(plan->h_dy[i]);
@@ -348,6 +351,11 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
         if ((e = cudaMemcpy(plan->d_fix, plan->pt.fix_table, fb, cudaMemcpyHostToDevice)) != cudaSuccess) return bail(e, "copy fixup table");
     }
     if ((e = cudaMalloc(&plan->d_hist, 64)) != cudaSuccess) return bail(e, "alloc hist");
+    const char* st_env = std::getenv("PLR_STATS");
+    if (st_env != nullptr && st_env[0] == '1') {
+        if ((e = cudaMalloc(&plan->d_stats, 64)) != cudaSuccess) return bail(e, "alloc stats");
+        if ((e = cudaMemset(plan->d_stats, 0, 64)) != cudaSuccess) return bail(e, "memset stats");
+    }
     if ((e = cudaMemset(plan->d_hist, 0, 64)) != cudaSuccess) return bail(e, "memset hist");
     *out = plan;
     return PLR_OK;
@@ -370,6 +378,17 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
                           (size_t)plan->pt.fixup_len * kAug * 4 + 64;
     info->ctas_per_sm = plan->ctas_per_sm;
     info->num_sms = plan->num_sms;
+    return PLR_OK;
+}
+
+plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out, int reset) {
+    if (plan == nullptr || out == nullptr) return fail(PLR_ERR_INVALID_ARG, "null argument");
+    if (plan->d_stats == nullptr) {
+        memset(out, 0, 8 * sizeof(uint64_t));
+        return PLR_OK;
+    }
+    CUDA_TRY(cudaMemcpy(out, plan->d_stats, 64, cudaMemcpyDeviceToHost), "stats copy");
+    if (reset) CUDA_TRY(cudaMemset(plan->d_stats, 0, 64), "stats reset");
     return PLR_OK;
 }
 

@@ -62,6 +62,7 @@ struct ScanParams {
     const T* y_hist;                     // k values y_{-k}..y_{-1} or null
     T* y_tail;                           // k slots y_{n-k}..y_{n-1} or null
     const A* lane_T;                     // [k*k][32]: T(X*l) per lane
+    unsigned long long* stats;           // debug counters (PLR_STATS=1) or null
     Tables<T, A> tab;
 };
 

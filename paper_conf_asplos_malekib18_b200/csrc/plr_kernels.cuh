@@ -328,11 +328,19 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 // once; the look-back is a single hop
                 A v[K];
                 if (lane == 0) {
-                    while (read_status<A, K>(prm.status, j - 1, v, tagA, tagI) != 2) __nanosleep(20);
+                    int ns = 16;
+                    while (read_status<A, K>(prm.status, j - 1, v, tagA, tagI) != 2) {
+                        __nanosleep(ns);
+                        ns = ns < 256 ? 2 * ns : ns;
+                    }
                 }
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = shfl_idx(lane == 0 ? v[q] : A(0), 0);
             } else {
+                // generic look-back: start once the tile's own aggregate is
+                // published, so the predecessors of the same wave have had
+                // the same time to publish theirs
+                mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
                 A acc[K];
                 A Tacc[K * kMaxK];
 #pragma unroll
@@ -343,8 +351,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 }
                 long long base = j - 1;
                 int tpl = 1;                       // first window: 32 tiles, then 32*kTPL
-                int spins = 0;
+                unsigned long long n_win = 0, n_wait = 0;
                 for (;;) {
+                    n_win++;
                     // lane owns tiles base - lane*tpl - t, t < tpl (contiguous)
                     A v[kTPL][K];
                     int st[kTPL];
@@ -362,19 +371,31 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
                     for (int t = kTPL - 1; t >= 0; t--)
                         if (t < tpl && st[t] == 2) first_incl = t;
-                    bool ready = true;
+                    int first_nr = kTPL;                         // first not-ready tile of the lane
 #pragma unroll
-                    for (int t = 0; t < kTPL; t++)
-                        if (t < tpl && t <= first_incl && st[t] == 0) ready = false;
+                    for (int t = kTPL - 1; t >= 0; t--)
+                        if (t < tpl && t <= first_incl && st[t] == 0) first_nr = t;
                     const unsigned incl = __ballot_sync(0xffffffffu, first_incl < tpl);
                     const int dl = incl ? (__ffs(incl) - 1) : 32;
                     const unsigned need = dl >= 31 ? 0xffffffffu : ((2u << dl) - 1u);
-                    const unsigned notready = __ballot_sync(0xffffffffu, !ready);
-                    if (notready & need) {                       // re-poll the window
-                        if (++spins > 4) __nanosleep(32);
+                    const unsigned notready = __ballot_sync(0xffffffffu, first_nr < kTPL) & need;
+                    if (notready) {
+                        // wait for the nearest not-ready tile alone, then re-read the window
+                        n_wait++;
+                        const int wl = __ffs(notready) - 1;
+                        const int wt = shfl_idx(first_nr, wl);
+                        if (lane == 0) {
+                            const long long jj = base - (long long)wl * tpl - wt;
+                            A tmp[K];
+                            int ns = 16;
+                            while (read_status<A, K>(prm.status, jj, tmp, tagA, tagI) == 0) {
+                                __nanosleep(ns);
+                                ns = ns < 256 ? 2 * ns : ns;
+                            }
+                        }
+                        __syncwarp();
                         continue;
                     }
-                    spins = 0;
                     // per-lane Horner fold over its tiles (up to its first inclusive)
                     const int last = (lane < dl) ? tpl - 1 : (lane == dl ? first_incl : -1);
                     A r[K];
@@ -404,7 +425,15 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
                     for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
                     matvec_acc<A, K>(acc, Tacc, R);
-                    if (dl < 32) break;
+                    if (dl < 32) {
+                        if (prm.stats != nullptr && lane == 0) {
+                            atomicAdd(&prm.stats[0], 1ull);                          // look-backs
+                            atomicAdd(&prm.stats[1], n_win);                         // windows read
+                            atomicAdd(&prm.stats[2], n_wait);                        // waits on a tile
+                            atomicAdd(&prm.stats[3], (unsigned long long)(j - (base - (long long)dl * tpl)));  // depth
+                        }
+                        break;
+                    }
                     // the next window lies 32*tpl tiles further back: Tacc *= T(32 tpl m)
                     const A* Tw = (tpl == 1) ? tb.Tw1 : tb.Tw8;
                     A nt[K * kMaxK];
@@ -428,7 +457,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 for (int q = 0; q < K; q++) Gp[q] = acc[q];
             }
             // the tile's own aggregate (phase A) is needed for its inclusive carry
-            mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
+            if (j == 0 || prm.decay) mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
             if (lane == 0) {
 #pragma unroll
                 for (int q = 0; q < K; q++) sG[slot * kMaxK + q] = Gp[q];

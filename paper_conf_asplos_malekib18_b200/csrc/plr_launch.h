@@ -21,6 +21,7 @@ struct LaunchArgs {
     const void* y_hist;
     void* y_tail;
     const void* lane_T;
+    unsigned long long* stats = nullptr;
     int grid;
     bool store;
     cudaStream_t stream;

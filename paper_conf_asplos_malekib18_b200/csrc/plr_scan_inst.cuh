@@ -36,6 +36,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     prm.y_hist = static_cast<const T*>(la.y_hist);
     prm.y_tail = static_cast<T*>(la.y_tail);
     prm.lane_T = static_cast<const A*>(la.lane_T);
+    prm.stats = la.stats;
     prm.tab = tab;
     kern<<<la.grid, (kW + 2) * 32, smem, la.stream>>>(prm);
     return cudaGetLastError();

@@ -111,17 +111,16 @@ def test_continue_chunks(cuda_plr, sig):
     plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
     xd = torch.from_numpy(x).cuda()
     yd = torch.empty_like(xd)
-    cuts = [0, 5, 4096, 4100, 20 * M + 8, 20 * M + 12, n]
+    cuts = [0, 4, 4096, 4100, 20 * M + 8, 20 * M + 12, n]     # chunk starts stay 16-byte aligned
+
+    def hist(t, s, L):
+        if s == 0 or L == 0:
+            return None
+        if s >= L:
+            return t[s - L:s]
+        return torch.cat([torch.zeros(L - s, dtype=t.dtype, device="cuda"), t[:s]])
     for s, e in zip(cuts[:-1], cuts[1:]):
-        xh = xd[s - sig.p:s] if (sig.p and s >= sig.p) else None
-        yh = yd[s - sig.k:s] if s >= sig.k else None
-        if s > 0 and (xh is None and sig.p) or (s > 0 and yh is None):
-            # histories that reach before index 0: pad with zeros
-            xh = torch.cat([torch.zeros(max(0, sig.p - s), dtype=xd.dtype, device="cuda"), xd[max(0, s - sig.p):s]]) if sig.p else None
-            yh = torch.cat([torch.zeros(max(0, sig.k - s), dtype=xd.dtype, device="cuda"), yd[max(0, s - sig.k):s]])
-        if s == 0:
-            xh, yh = None, None
-        plan.continue_(xd[s:e], yd[s:e], x_hist=xh, y_hist=yh)
+        plan.continue_(xd[s:e], yd[s:e], x_hist=hist(xd, s, sig.p), y_hist=hist(yd, s, sig.k))
     check(yd.cpu().numpy(), ref, sig.dtype, sig.name)
 
 
