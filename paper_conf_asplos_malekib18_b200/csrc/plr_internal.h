@@ -19,7 +19,7 @@ constexpr int kMaxX = 31;
 constexpr int kMaxW = 16;
 constexpr int kStatusWords = 4;     // u64 status words per tile (>= kMaxK)
 constexpr int kAug = 8;             // augmented state slots: x_{-4..-1}, y_{-4..-1}
-constexpr int kTPL = 8;             // look-back: tiles per lane in a wide window
+constexpr int kTPL = 8;             // look-back: tiles per lane in a wide window (2^3)
 
 struct Geometry {
     int X, W, S;
@@ -41,10 +41,7 @@ struct Tables {
     A Tblk[4][kMaxK * kMaxK];            // T(32 X * 2^s)       warp-aggregate scan
     A Twin[kMaxW][kMaxK * kMaxK];        // T(32 X * w)         warp carry-in
     A Tm[kMaxK * kMaxK];                 // T(m)                inclusive = agg + T(m) G
-    A Tlb1[5][kMaxK * kMaxK];            // T(m * 2^s)          narrow window fold
-    A Tlb8[5][kMaxK * kMaxK];            // T(kTPL m * 2^s)     wide window fold
-    A Tw1[kMaxK * kMaxK];                // T(32 m)             next narrow window
-    A Tw8[kMaxK * kMaxK];                // T(32 kTPL m)        next wide window
+    A Tpow[9][kMaxK * kMaxK];            // T(m * 2^s), s <= 8  look-back folds and skips
 };
 
 template <typename T, typename A>

@@ -337,9 +337,14 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = shfl_idx(lane == 0 ? v[q] : A(0), 0);
             } else {
-                // generic look-back: start once the tile's own aggregate is
-                // published, so the predecessors of the same wave have had
-                // the same time to publish theirs
+                // generic look-back: fold the tiles
+                // j-1, j-2, ... nearest first, G_{j-1} = sum_d T(d m) v_{j-1-d},
+                // v = aggregate for "P" tiles and the inclusive carry of the
+                // first "I" tile.  Each poll folds the ready prefix of its
+                // window (up to the first not-ready or first inclusive tile)
+                // and never re-reads folded tiles.  Start once the tile's own
+                // aggregate is published: the predecessors of the same wave
+                // have had the same time to publish theirs.
                 mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
                 A acc[K];
                 A Tacc[K * kMaxK];
@@ -349,109 +354,99 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
                     for (int r = 0; r < kMaxK; r++) Tacc[q * kMaxK + r] = (q == r) ? A(1) : A(0);
                 }
-                long long base = j - 1;
-                int tpl = 1;                       // first window: 32 tiles, then 32*kTPL
+                long long o = 0;                   // distance of the first unfolded tile from j-1
+                int ltpl = 1;                      // log2 tiles per lane: 2 (64-tile window), then 8
+                int ns = 32;
                 unsigned long long n_win = 0, n_wait = 0;
                 for (;;) {
                     n_win++;
-                    // lane owns tiles base - lane*tpl - t, t < tpl (contiguous)
+                    const int tpl = 1 << ltpl;
                     A v[kTPL][K];
                     int st[kTPL];
-                    int first_incl = kTPL;
 #pragma unroll
                     for (int t = 0; t < kTPL; t++) {
                         st[t] = 2;
 #pragma unroll
                         for (int q = 0; q < K; q++) v[t][q] = A(0);
                         if (t < tpl) {
-                            const long long jj = base - (long long)lane * tpl - t;
+                            const long long jj = j - 1 - (o + (long long)lane * tpl + t);
                             if (jj >= 0) st[t] = read_status<A, K>(prm.status, jj, v[t], tagA, tagI);
                         }
                     }
-#pragma unroll
-                    for (int t = kTPL - 1; t >= 0; t--)
-                        if (t < tpl && st[t] == 2) first_incl = t;
-                    int first_nr = kTPL;                         // first not-ready tile of the lane
-#pragma unroll
-                    for (int t = kTPL - 1; t >= 0; t--)
-                        if (t < tpl && t <= first_incl && st[t] == 0) first_nr = t;
-                    const unsigned incl = __ballot_sync(0xffffffffu, first_incl < tpl);
-                    const int dl = incl ? (__ffs(incl) - 1) : 32;
-                    const unsigned need = dl >= 31 ? 0xffffffffu : ((2u << dl) - 1u);
-                    const unsigned notready = __ballot_sync(0xffffffffu, first_nr < kTPL) & need;
-                    if (notready) {
-                        // wait for the nearest not-ready tile alone, then re-read the window
-                        n_wait++;
-                        const int wl = __ffs(notready) - 1;
-                        const int wt = shfl_idx(first_nr, wl);
-                        if (lane == 0) {
-                            const long long jj = base - (long long)wl * tpl - wt;
-                            A tmp[K];
-                            int ns = 16;
-                            while (read_status<A, K>(prm.status, jj, tmp, tagA, tagI) == 0) {
-                                __nanosleep(ns);
-                                ns = ns < 256 ? 2 * ns : ns;
-                            }
-                        }
-                        __syncwarp();
-                        continue;
-                    }
-                    // per-lane Horner fold over its tiles (up to its first inclusive)
-                    const int last = (lane < dl) ? tpl - 1 : (lane == dl ? first_incl : -1);
-                    A r[K];
-#pragma unroll
-                    for (int q = 0; q < K; q++) r[q] = A(0);
+                    int fi = kTPL, fn = kTPL;                    // first inclusive / not-ready in lane
 #pragma unroll
                     for (int t = kTPL - 1; t >= 0; t--) {
-                        if (t <= last) {
-                            A nr[K];
-#pragma unroll
-                            for (int q = 0; q < K; q++) nr[q] = v[t][q];
-                            matvec_acc<A, K>(nr, tb.Tm, r);
-#pragma unroll
-                            for (int q = 0; q < K; q++) r[q] = nr[q];
-                        }
+                        if (t < tpl && st[t] == 2) fi = t;
+                        if (t < tpl && st[t] == 0) fn = t;
                     }
-                    // tree over lanes: R = sum_l T(l * tpl * m) r_l
-                    const A* Tl5 = (tpl == 1) ? &tb.Tlb1[0][0] : &tb.Tlb8[0][0];
+                    const unsigned bi = __ballot_sync(0xffffffffu, fi < tpl);
+                    const unsigned bn = __ballot_sync(0xffffffffu, fn < tpl);
+                    const int dI = bi ? (__ffs(bi) - 1) * tpl + shfl_idx(fi, __ffs(bi) - 1) : 1 << 30;
+                    const int dN = bn ? (__ffs(bn) - 1) * tpl + shfl_idx(fn, __ffs(bn) - 1) : 1 << 30;
+                    const bool found = dI < dN;
+                    const int e = found ? dI + 1 : (bn ? dN : 32 * tpl);   // tiles to fold now
+                    if (e > 0) {
+                        // per-lane Horner over its tiles with window offset < e
+                        A r[K];
 #pragma unroll
-                    for (int s2 = 0; s2 < 5; s2++) {
-                        A o[K];
+                        for (int q = 0; q < K; q++) r[q] = A(0);
 #pragma unroll
-                        for (int q = 0; q < K; q++) o[q] = shfl_down(r[q], 1 << s2);
-                        matvec_acc<A, K>(r, Tl5 + s2 * kMaxK * kMaxK, o);
-                    }
-                    A R[K];
+                        for (int t = kTPL - 1; t >= 0; t--) {
+                            if (t < tpl && lane * tpl + t < e) {
+                                A nr[K];
 #pragma unroll
-                    for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
-                    matvec_acc<A, K>(acc, Tacc, R);
-                    if (dl < 32) {
-                        if (prm.stats != nullptr && lane == 0) {
-                            atomicAdd(&prm.stats[0], 1ull);                          // look-backs
-                            atomicAdd(&prm.stats[1], n_win);                         // windows read
-                            atomicAdd(&prm.stats[2], n_wait);                        // waits on a tile
-                            atomicAdd(&prm.stats[3], (unsigned long long)(j - (base - (long long)dl * tpl)));  // depth
+                                for (int q = 0; q < K; q++) nr[q] = v[t][q];
+                                matvec_acc<A, K>(nr, tb.Tm, r);
+#pragma unroll
+                                for (int q = 0; q < K; q++) r[q] = nr[q];
+                            }
                         }
-                        break;
-                    }
-                    // the next window lies 32*tpl tiles further back: Tacc *= T(32 tpl m)
-                    const A* Tw = (tpl == 1) ? tb.Tw1 : tb.Tw8;
-                    A nt[K * kMaxK];
+                        // tree over lanes: R = sum_l T(l tpl m) r_l, T(tpl m 2^s) = Tpow[ltpl + s]
 #pragma unroll
-                    for (int q = 0; q < K; q++)
+                        for (int s2 = 0; s2 < 5; s2++) {
+                            A o2[K];
 #pragma unroll
-                        for (int c2 = 0; c2 < K; c2++) {
-                            A a2 = A(0);
-#pragma unroll
-                            for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], Tw[t * kMaxK + c2], a2);
-                            nt[q * kMaxK + c2] = a2;
+                            for (int q = 0; q < K; q++) o2[q] = shfl_down(r[q], 1 << s2);
+                            matvec_acc<A, K>(r, tb.Tpow[ltpl + s2], o2);
                         }
+                        A R[K];
 #pragma unroll
-                    for (int q = 0; q < K; q++)
+                        for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
+                        matvec_acc<A, K>(acc, Tacc, R);
+                        if (found) break;
+                        // skip the folded tiles: Tacc *= T(e m) (binary powers)
+#pragma unroll 1
+                        for (int s2 = 0; s2 < 9; s2++) {
+                            if (!((e >> s2) & 1)) continue;
+                            A nt[K * kMaxK];
 #pragma unroll
-                        for (int c2 = 0; c2 < K; c2++) Tacc[q * kMaxK + c2] = nt[q * kMaxK + c2];
-                    base -= 32LL * tpl;
-                    tpl = kTPL;
+                            for (int q = 0; q < K; q++)
+#pragma unroll
+                                for (int c2 = 0; c2 < K; c2++) {
+                                    A a2 = A(0);
+#pragma unroll
+                                    for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], tb.Tpow[s2][t * kMaxK + c2], a2);
+                                    nt[q * kMaxK + c2] = a2;
+                                }
+#pragma unroll
+                            for (int q = 0; q < K; q++)
+#pragma unroll
+                                for (int c2 = 0; c2 < K; c2++) Tacc[q * kMaxK + c2] = nt[q * kMaxK + c2];
+                        }
+                        o += e;
+                        ns = 32;
+                        if (!bn) ltpl = 3;                         // nothing pending: widen to 256 tiles
+                    } else {
+                        n_wait++;                                  // nearest tile not ready yet
+                        __nanosleep(ns);
+                        ns = ns < 512 ? 2 * ns : ns;
+                    }
+                }
+                if (prm.stats != nullptr && lane == 0) {
+                    atomicAdd(&prm.stats[0], 1ull);                // look-backs
+                    atomicAdd(&prm.stats[1], n_win);               // window polls
+                    atomicAdd(&prm.stats[2], n_wait);              // polls that folded nothing
+                    atomicAdd(&prm.stats[3], (unsigned long long)(o + 1));  // depth folded (approx.)
                 }
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = acc[q];

@@ -95,10 +95,7 @@ void fill_tables(const Mat<R>& M, int k, Geometry geo, Tables<T, A>* tb, A* lane
     for (int s = 0; s < 4; s++) store_mat(mpow(M, (32 * X) << s), tb->Tblk[s], cvtA);
     for (int w = 0; w < kMaxW; w++) store_mat(mpow(M, 32 * X * (uint64_t)w), tb->Twin[w], cvtA);
     store_mat(mpow(M, m), tb->Tm, cvtA);
-    for (int s = 0; s < 5; s++) store_mat(mpow(M, m << s), tb->Tlb1[s], cvtA);
-    for (int s = 0; s < 5; s++) store_mat(mpow(M, (kTPL * m) << s), tb->Tlb8[s], cvtA);
-    store_mat(mpow(M, 32 * m), tb->Tw1, cvtA);
-    store_mat(mpow(M, 32 * kTPL * m), tb->Tw8, cvtA);
+    for (int s = 0; s < 9; s++) store_mat(mpow(M, m << s), tb->Tpow[s], cvtA);
     for (int l = 0; l < 32; l++) {
         Mat<R> Tl = mpow(M, X * (uint64_t)l);
         for (int q = 0; q < k; q++)
