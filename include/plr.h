@@ -135,7 +135,9 @@ plr_status plr_execute_continue(plr_plan* plan, const void* x, void* y, size_t n
 /* Reduce-only pass: the end state of x[0..n) with zero history, without
  * writing y (reads n elements).  payload (device, PLR_PAYLOAD_BYTES) gets
  *   uint64 n | uint32 x_tail[4] (x_{n-4}..x_{n-1}) | uint32 y_tail[4] (y_{n-4}..y_{n-1})
- * (bit patterns of the dtype; indices < 0 are 0).  This is a segment's
+ * (bit patterns of the dtype; indices < 0 are 0; plr_reduce fills only the
+ * last k y slots, the others stay 0 and are never read by the combine's
+ * order-k recurrence row).  This is a segment's
  * contribution to the sharded combine. */
 plr_status plr_reduce(plr_plan* plan, const void* x, size_t n, void* payload, void* stream);
 

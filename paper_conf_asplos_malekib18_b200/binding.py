@@ -5,7 +5,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libplr_b200.so")
+LIB_PATH = os.environ.get("PLR_LIB") or os.path.join(_HERE, "libplr_b200.so")   # PLR_LIB: experiment variants
 PAYLOAD_BYTES = 64
 
 if not os.path.exists(LIB_PATH):

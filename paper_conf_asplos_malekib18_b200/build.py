@@ -15,14 +15,19 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-BUILD = os.path.join(HERE, "_build")
-LIB = os.path.join(HERE, "libplr_b200.so")
+# experiment variants: PLR_VARIANT="STAGES,LAG" builds libplr_b200_sS_dD.so
+_VAR = os.environ.get("PLR_VARIANT")
+_SUFFIX = "" if not _VAR else "_s%s_d%s" % tuple(_VAR.split(","))
+BUILD = os.path.join(HERE, "_build" + _SUFFIX)
+LIB = os.path.join(HERE, "libplr_b200%s.so" % _SUFFIX)
 INCLUDE = os.path.join(os.path.dirname(HERE), "include")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUDE, "-I" + CSRC,
           "--ftz=true", "--prec-div=true", "--prec-sqrt=true", "--fmad=true"]
+if _VAR:
+    COMMON += ["-DPLR_STAGES=%s" % _VAR.split(",")[0], "-DPLR_LAG=%s" % _VAR.split(",")[1]]
 
 
 def _sources():

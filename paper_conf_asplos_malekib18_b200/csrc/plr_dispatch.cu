@@ -3,10 +3,14 @@
 
 namespace plr {
 
+#ifndef PLR_STAGES
+#define PLR_STAGES 5
+#endif
+
 Geometry default_geometry(plr_dtype, int, int) {
     // x = 15 elements per thread (odd: conflict-free strided smem access),
-    // 8 compute warps, 4-stage TMA ring: m = 3840 elements = 15 KB per tile.
-    return Geometry{15, 8, 4};
+    // 8 compute warps, PLR_STAGES-stage TMA ring: m = 3840 elements = 15 KB per tile.
+    return Geometry{15, 8, PLR_STAGES};
 }
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la) {

@@ -202,29 +202,31 @@ __device__ __forceinline__ int read_status(const unsigned long long* status, lon
 }
 
 // ------------------------------------------------------ shared memory ------
-template <typename T, typename A, int K, int X, int W, int S>
+template <typename T, typename A, int K, int X, int W, int S, int D>
 struct Layout {
+    static constexpr int NS = D + 1;                            // pipeline slots (tiles between A and B)
     static constexpr int M = 32 * W * X;
     static constexpr int NC = 32 * W;
     static constexpr int SW = M + kHalo;                        // words per stage
     static constexpr size_t off_stage = 0;
-    static constexpr size_t off_E = (size_t)S * SW * sizeof(T);                       // [2][K][NC] A
-    static constexpr size_t off_Pw = off_E + 2 * (size_t)K * NC * sizeof(A);          // [2][W][K] A
-    static constexpr size_t off_At = off_Pw + 2 * (size_t)W * K * sizeof(A);          // [2][K] A
-    static constexpr size_t off_G = off_At + 2 * (size_t)kMaxK * sizeof(A);           // [2][K] A
-    static constexpr size_t off_wagg = off_G + 2 * (size_t)kMaxK * sizeof(A);         // [2][W][K] A
-    static constexpr size_t off_bar = (off_wagg + 2 * (size_t)W * kMaxK * sizeof(A) + 15) & ~(size_t)15;
-    // bars: full[S], done[S], agg[2], carry[2]
-    static constexpr size_t off_tile = off_bar + (2 * S + 4) * 8;                    // tile_of[S]
-    static constexpr size_t off_aggtile = off_tile + S * 8;                           // agg_tile[2]
-    static constexpr size_t bytes = off_aggtile + 2 * 8;
+    static constexpr size_t off_E = (size_t)S * SW * sizeof(T);                       // [NS][K][NC] A
+    static constexpr size_t off_Pw = off_E + NS * (size_t)K * NC * sizeof(A);         // [NS][W][K] A
+    static constexpr size_t off_At = off_Pw + NS * (size_t)W * K * sizeof(A);         // [NS][K] A
+    static constexpr size_t off_G = off_At + NS * (size_t)kMaxK * sizeof(A);          // [NS][K] A
+    static constexpr size_t off_wagg = off_G + NS * (size_t)kMaxK * sizeof(A);        // [NS][W][K] A
+    static constexpr size_t off_bar = (off_wagg + NS * (size_t)W * kMaxK * sizeof(A) + 15) & ~(size_t)15;
+    // bars: full[S], done[S], agg[NS], carry[NS]
+    static constexpr size_t off_tile = off_bar + (2 * S + 2 * NS) * 8;               // tile_of[S]
+    static constexpr size_t off_aggtile = off_tile + S * 8;                           // agg_tile[NS]
+    static constexpr size_t bytes = off_aggtile + NS * 8;
 };
 
 // ------------------------------------------------------ the scan kernel ----
-template <typename T, typename A, int K, int P, int X, int W, int S, bool STORE>
+template <typename T, typename A, int K, int P, int X, int W, int S, int D, bool STORE>
 __global__ void __launch_bounds__((W + 2) * 32)
 plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
-    using L = Layout<T, A, K, X, W, S>;
+    using L = Layout<T, A, K, X, W, S, D>;
+    constexpr int NS = L::NS;
     constexpr int M = L::M;
     constexpr int SW = L::SW;
     constexpr int NC = L::NC;
@@ -234,7 +236,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     static_assert(P <= kHalo, "halo");
     using SIO = StatusIO<A>;
     static_assert(K * SIO::kWords <= 2 * kStatusWords, "status words");
-    static_assert(S >= 3, "phase B of tile i runs after phase A of tile i+1: needs >= 3 stages");
+    static_assert(D >= 1 && S >= D + 2, "phase B of tile i runs after phase A of tile i+D: needs S >= D+2 stages");
 
     extern __shared__ __align__(128) unsigned char smem[];
     T* stages = reinterpret_cast<T*>(smem + L::off_stage);
@@ -246,7 +248,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     uint64_t* full_bar = reinterpret_cast<uint64_t*>(smem + L::off_bar);
     uint64_t* done_bar = full_bar + S;
     uint64_t* agg_bar = done_bar + S;
-    uint64_t* carry_bar = agg_bar + 2;
+    uint64_t* carry_bar = agg_bar + NS;
     long long* tile_of = reinterpret_cast<long long*>(smem + L::off_tile);
     long long* agg_tile = reinterpret_cast<long long*>(smem + L::off_aggtile);
 
@@ -259,7 +261,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 
     if (tid == 0) {
         for (int s = 0; s < S; s++) { mbar_init(&full_bar[s], 1); mbar_init(&done_bar[s], NC); }
-        for (int s = 0; s < 2; s++) { mbar_init(&agg_bar[s], 1); mbar_init(&carry_bar[s], 1); }
+        for (int s = 0; s < NS; s++) { mbar_init(&agg_bar[s], 1); mbar_init(&carry_bar[s], 1); }
         fence_mbar_init();
     }
     __syncthreads();
@@ -315,7 +317,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
         for (int it = 0;; it++) {
             const int s = it % S;
-            const int slot = it & 1;
+            const int slot = it % NS;
             mbar_wait(&full_bar[s], (uint32_t)((it / S) & 1));
             const long long j = tile_of[s];
             if (j >= ntiles) break;
@@ -345,7 +347,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 // and never re-reads folded tiles.  Start once the tile's own
                 // aggregate is published: the predecessors of the same wave
                 // have had the same time to publish theirs.
-                mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
+                mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
                 A acc[K];
                 A Tacc[K * kMaxK];
 #pragma unroll
@@ -452,7 +454,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 for (int q = 0; q < K; q++) Gp[q] = acc[q];
             }
             // the tile's own aggregate (phase A) is needed for its inclusive carry
-            if (j == 0 || prm.decay) mbar_wait(&agg_bar[slot], (uint32_t)((it >> 1) & 1));
+            if (j == 0 || prm.decay) mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
             if (lane == 0) {
 #pragma unroll
                 for (int q = 0; q < K; q++) sG[slot * kMaxK + q] = Gp[q];
@@ -481,7 +483,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // phase A of pipeline iteration `it`: returns the tile id (>= ntiles: stop)
     auto phaseA = [&](int it) -> long long {
         const int s = it % S;
-        const int slot = it & 1;
+        const int slot = it % NS;
         mbar_wait(&full_bar[s], (uint32_t)((it / S) & 1));
         const long long j = tile_of[s];
         if (j >= ntiles) {
@@ -576,8 +578,8 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             for (int q = 0; q < K; q++) At[q] = shfl_idx(u_[q], W - 1);
             publish_status<A, K>(prm.status, j, At, prm.decay ? 2u * prm.epoch + 1u : 2u * prm.epoch, lane);
         }
-        // wagg is double-buffered by slot: its next writer (tile it+2) runs
-        // after every warp passed tile it+1's barrier
+        // wagg is buffered per slot: its next writer (tile it+NS) runs after
+        // every warp passed tile it+1's barrier
         __syncwarp();                                           // sPw (lane 0) visible to the warp
         if (tid == 0) { agg_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
         return j;
@@ -586,8 +588,8 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // phase B of pipeline iteration `it` (tile id j)
     auto phaseB = [&](int it, long long j) {
         const int s = it % S;
-        const int slot = it & 1;
-        mbar_wait(&carry_bar[slot], (uint32_t)((it >> 1) & 1));
+        const int slot = it % NS;
+        mbar_wait(&carry_bar[slot], (uint32_t)((it / NS) & 1));
         const bool ragged = (j == ntiles - 1) && last_ragged;
         T* st = stages + (size_t)s * SW;
         const long long g0 = j * (long long)M + (long long)tid * X;
@@ -643,14 +645,21 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         mbar_arrive(&done_bar[s]);
     };
 
-    long long jprev = phaseA(0);
-    if (jprev >= ntiles) return;
-    for (int it = 1;; it++) {
-        const long long j = phaseA(it);
-        phaseB(it - 1, jprev);
-        if (j >= ntiles) break;
-        jprev = j;
+    // software pipeline: phase A runs D tiles ahead of phase B
+    long long jq[NS];
+    int na = 0, nb = 0;                             // phases A / B done
+    for (; na < D; na++) {
+        jq[na % NS] = phaseA(na);
+        if (jq[na % NS] >= ntiles) break;
     }
+    for (bool stop = na < D; !stop;) {
+        const long long j = phaseA(na);
+        jq[na % NS] = j;
+        phaseB(nb, jq[nb % NS]);
+        nb++;
+        if (j >= ntiles) stop = true; else na++;
+    }
+    for (; nb < na; nb++) phaseB(nb, jq[nb % NS]);   // drain
 }
 
 }  // namespace dev

@@ -8,12 +8,18 @@
 namespace plr {
 namespace inst {
 
-constexpr int kX = 15, kW = 8, kS = 4;   // see default_geometry()
+#ifndef PLR_STAGES
+#define PLR_STAGES 5
+#endif
+#ifndef PLR_LAG
+#define PLR_LAG 2
+#endif
+constexpr int kX = 15, kW = 8, kS = PLR_STAGES, kD = PLR_LAG;   // see default_geometry()
 
 template <typename T, typename A, int K, int P, bool STORE>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
-    auto kern = &dev::plr_scan_kernel<T, A, K, P, kX, kW, kS, STORE>;
-    const size_t smem = dev::Layout<T, A, K, kX, kW, kS>::bytes;
+    auto kern = &dev::plr_scan_kernel<T, A, K, P, kX, kW, kS, kD, STORE>;
+    const size_t smem = dev::Layout<T, A, K, kX, kW, kS, kD>::bytes;
     static bool configured = false;
     if (!configured) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

@@ -153,8 +153,9 @@ def test_reduce_payload_and_combine(cuda_plr, sig):
         got = pl.cpu().numpy()
         assert int(got[:8].view(np.uint64)[0]) == nr
         npdt = np.int32 if sig.dtype == "int32" else np.float32
-        yt = got[24:40].view(npdt)[4 - min(4, nr):]
-        check(yt.astype(np.float64) if sig.dtype == "float32" else yt, yz[-4:], sig.dtype, "payload %d" % r)
+        kk = min(sig.k if not decay else 4, nr)       # plr_reduce fills the last k outputs only
+        yt = got[24:40].view(npdt)[4 - kk:]
+        check(yt.astype(np.float64) if sig.dtype == "float32" else yt, yz[len(yz) - kk:], sig.dtype, "payload %d" % r)
         pls.append(pl)
     payloads = torch.cat(pls)
     host_pl = payloads.cpu().numpy().tobytes()
