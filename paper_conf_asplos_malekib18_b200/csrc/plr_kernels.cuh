@@ -18,10 +18,10 @@
 //   a7 store
 // Roles: warp W (producer) takes tickets and moves whole tiles with TMA bulk
 // copies (cp.async.bulk + mbarrier complete_tx) into an S-stage shared-memory
-// ring and back out with TMA bulk stores; warp W+1 (look-back) runs a5 for
-// the CTA's tiles in order; warps 0..W-1 (compute) run phase A (a1-a4) of
-// tile i+1 before phase B (a6-a7) of tile i, so the look-back latency of a
-// tile overlaps a whole tile of compute.
+// ring and back out with TMA bulk stores; warps W+1..W+NL (look-back) run a5
+// for the CTA's tiles, taking turns; warps 0..W-1 (compute) run phase A
+// (a1-a4) of tile i+D before phase B (a6-a7) of tile i, so the look-back
+// latency of a tile overlaps D tiles of compute.
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
@@ -222,8 +222,8 @@ struct Layout {
 };
 
 // ------------------------------------------------------ the scan kernel ----
-template <typename T, typename A, int K, int P, int X, int W, int S, int D, bool STORE>
-__global__ void __launch_bounds__((W + 2) * 32)
+template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool STORE>
+__global__ void __launch_bounds__((W + 1 + NL) * 32)
 plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = Layout<T, A, K, X, W, S, D>;
     constexpr int NS = L::NS;
@@ -237,6 +237,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using SIO = StatusIO<A>;
     static_assert(K * SIO::kWords <= 2 * kStatusWords, "status words");
     static_assert(D >= 1 && S >= D + 2, "phase B of tile i runs after phase A of tile i+D: needs S >= D+2 stages");
+    static_assert(NL >= 1 && NL <= S, "look-back warps");
 
     extern __shared__ __align__(128) unsigned char smem[];
     T* stages = reinterpret_cast<T*>(smem + L::off_stage);
@@ -270,11 +271,19 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     if (warp == W) {
         if (lane != 0) return;
         const uint64_t pol = policy_evict_first();
-        bool done = false;
-        auto fill = [&](int s) {
+        int fills = 0;                                  // pipeline index of the next fill
+        int stop_at = 1 << 30;                          // pipeline index of the first stop marker
+        auto fill = [&]() {
+            const int idx = fills++;
+            const int s = idx % S;
+            if (idx > stop_at) {                        // extra stop markers for the look-back warps
+                tile_of[s] = ntiles;
+                mbar_arrive(&full_bar[s]);
+                return;
+            }
             const long long j = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
             tile_of[s] = j;
-            if (j >= ntiles) { done = true; mbar_arrive(&full_bar[s]); return; }
+            if (j >= ntiles) { stop_at = idx; mbar_arrive(&full_bar[s]); return; }
             if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_bar[s]); return; }   // compute loads it
             T* st = stages + (size_t)s * SW;
             if (j == 0) {
@@ -288,7 +297,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 bulk_load(st, prm.x + (size_t)j * M - kHalo, SW * sizeof(T), &full_bar[s], pol);
             }
         };
-        for (int s = 0; s < S && !done; s++) fill(s);
+        // every look-back warp must see a stop marker: NL of them after the last tile
+        auto more = [&]() { return fills < stop_at + NL; };
+        for (int s = 0; s < S && more(); s++) fill();
         for (int it = 0;; it++) {
             const int s = it % S;
             const long long j = tile_of[s];
@@ -300,9 +311,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 bulk_commit();
                 stored = true;
             }
-            if (it >= 1 && !done) {
+            if (it >= 1 && more()) {
                 if (stored) bulk_wait_read<1>(); else bulk_wait_read<0>();
-                fill((it - 1) % S);
+                fill();                                 // stage (it-1) % S, pipeline index it-1+S
             }
         }
         bulk_wait_all<0>();
@@ -313,9 +324,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // Runs a5 for the CTA's tiles in ticket order.  It learns the tile id from
     // the full barrier (as soon as the tile is loaded) and walks back without
     // waiting for the tile's own aggregate, which the compute warps publish.
-    if (warp == W + 1) {
+    if (warp > W) {
         const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
-        for (int it = 0;; it++) {
+        for (int it = warp - (W + 1);; it += NL) {     // NL look-back warps take turns
             const int s = it % S;
             const int slot = it % NS;
             mbar_wait(&full_bar[s], (uint32_t)((it / S) & 1));

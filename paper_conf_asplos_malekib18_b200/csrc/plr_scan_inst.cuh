@@ -14,11 +14,14 @@ namespace inst {
 #ifndef PLR_LAG
 #define PLR_LAG 2
 #endif
-constexpr int kX = 15, kW = 8, kS = PLR_STAGES, kD = PLR_LAG;   // see default_geometry()
+#ifndef PLR_NL
+#define PLR_NL 2
+#endif
+constexpr int kX = 15, kW = 8, kS = PLR_STAGES, kD = PLR_LAG, kNL = PLR_NL;   // see default_geometry()
 
 template <typename T, typename A, int K, int P, bool STORE>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
-    auto kern = &dev::plr_scan_kernel<T, A, K, P, kX, kW, kS, kD, STORE>;
+    auto kern = &dev::plr_scan_kernel<T, A, K, P, kX, kW, kS, kD, kNL, STORE>;
     const size_t smem = dev::Layout<T, A, K, kX, kW, kS, kD>::bytes;
     static bool configured = false;
     if (!configured) {
@@ -27,7 +30,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
         configured = true;
     }
     if (la.occupancy_out != nullptr)    // occupancy query: report CTAs/SM, do not launch
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, (kW + 2) * 32, smem);
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, (kW + 1 + kNL) * 32, smem);
     ScanParams<T, A> prm;
     prm.x = static_cast<const T*>(la.x);
     prm.y = static_cast<T*>(la.y);
@@ -44,7 +47,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     prm.lane_T = static_cast<const A*>(la.lane_T);
     prm.stats = la.stats;
     prm.tab = tab;
-    kern<<<la.grid, (kW + 2) * 32, smem, la.stream>>>(prm);
+    kern<<<la.grid, (kW + 1 + kNL) * 32, smem, la.stream>>>(prm);
     return cudaGetLastError();
 }
 

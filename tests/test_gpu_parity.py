@@ -137,17 +137,17 @@ def test_reduce_payload_and_combine(cuda_plr, sig):
     ref = oracle.recurrence(x, sig.a, sig.b, sig.dtype)
     plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
     decay = plan.info["cls"] == "DECAY"
-    xd = torch.from_numpy(x).cuda()
-    yd = torch.empty_like(xd)
     starts = np.cumsum([0] + sizes)
+    # each "rank" owns its segment in its own (aligned) allocation, as on a real box
+    xs = [torch.from_numpy(x[starts[r]:starts[r] + nr].copy()).cuda() for r, nr in enumerate(sizes)]
+    ys = [torch.empty_like(t) for t in xs]
     pls = []
     for r, nr in enumerate(sizes):
-        seg = xd[starts[r]:starts[r] + nr]
         if decay:
-            plan(seg, yd[starts[r]:starts[r] + nr])
-            pl = plan.payload_from_output(seg, yd[starts[r]:starts[r] + nr])
+            plan(xs[r], ys[r])
+            pl = plan.payload_from_output(xs[r], ys[r])
         else:
-            pl = plan.reduce(seg)
+            pl = plan.reduce(xs[r])
         # payload == oracle zero-history tails
         yz = oracle.recurrence(x[starts[r]:starts[r] + nr], sig.a, sig.b, sig.dtype)
         got = pl.cpu().numpy()
@@ -162,14 +162,12 @@ def test_reduce_payload_and_combine(cuda_plr, sig):
     for r, nr in enumerate(sizes):
         hist = plan.combine(payloads, r, len(sizes))
         assert hist.cpu().numpy().tobytes() == plan.combine_host(host_pl, r, len(sizes))
-        seg = xd[starts[r]:starts[r] + nr]
-        out = yd[starts[r]:starts[r] + nr]
         if decay:
-            plan.fixup(out, hist)
+            plan.fixup(ys[r], hist)
         else:
             xh = hist[4 - sig.p:4] if sig.p else None
-            plan.continue_(seg, out, x_hist=xh, y_hist=hist[8 - sig.k:8])
-    check(yd.cpu().numpy(), ref, sig.dtype, sig.name)
+            plan.continue_(xs[r], ys[r], x_hist=xh, y_hist=hist[8 - sig.k:8])
+    check(torch.cat(ys).cpu().numpy(), ref, sig.dtype, sig.name)
 
 
 @pytest.mark.parametrize("sig", [workloads.BY_NAME[n] for n in ("prefix", "order3", "hp3")], ids=lambda s: s.name)

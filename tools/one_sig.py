@@ -1,0 +1,18 @@
+"""Run one Table-1 signature a few times at n (default 2^30): profiling target."""
+import os
+import sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+import paper_conf_asplos_malekib18_b200 as plr  # noqa: E402
+import workloads  # noqa: E402
+
+name = sys.argv[1]
+n = int(sys.argv[2]) if len(sys.argv) > 2 else 1 << 30
+sig = workloads.BY_NAME[name]
+x = workloads.device_input(n, sig.dtype, 1)
+y = torch.empty_like(x)
+plan = plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+for _ in range(4):
+    plan(x, y)
+torch.cuda.synchronize()
+print("done", name, n)
