@@ -24,8 +24,11 @@ from .binding import (  # noqa: F401
     Plan,
     ShardComm,
     abi_version,
+    broadcast_bytes,
+    gather_payloads,
     lib,
     shard_bounds,
 )
 
-__all__ = ["Plan", "PLRError", "ShardComm", "shard_bounds", "lib", "LIB_PATH", "PAYLOAD_BYTES", "abi_version"]
+__all__ = ["Plan", "PLRError", "ShardComm", "shard_bounds", "broadcast_bytes", "gather_payloads", "lib",
+           "LIB_PATH", "PAYLOAD_BYTES", "abi_version"]

@@ -248,6 +248,26 @@ class Plan:
         return out
 
 
+def broadcast_bytes(payload, group=None) -> bytes:
+    """Group rank 0's bytes to every rank of `group` (torch.distributed)."""
+    import torch.distributed as dist
+    obj = [payload if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+    return obj[0]
+
+
+def gather_payloads(payload: bytes, group=None) -> bytes:
+    """All ranks' 64-byte payloads in rank order (host path over the process
+    group; the device path uses plr_execute_sharded's NCCL allgather)."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    mine = torch.frombuffer(bytearray(payload), dtype=torch.uint8)
+    out = [torch.empty(PAYLOAD_BYTES, dtype=torch.uint8) for _ in range(world)]
+    dist.all_gather(out, mine, group=group)
+    return b"".join(bytes(t.numpy().tobytes()) for t in out)
+
+
 class ShardComm:
     """NCCL communicator of the library, bootstrapped through torch.distributed:
     rank 0 creates the unique id, the process group broadcasts its bytes."""
@@ -259,9 +279,7 @@ class ShardComm:
         idbuf = ctypes.create_string_buffer(128)
         if self.rank == 0:
             _check(lib.plr_nccl_unique_id(idbuf, 128), "plr_nccl_unique_id")
-        obj = [idbuf.raw if self.rank == 0 else None]
-        dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
-        idbuf = ctypes.create_string_buffer(obj[0], 128)
+        idbuf = ctypes.create_string_buffer(broadcast_bytes(idbuf.raw, group), 128)
         h = _P()
         _check(lib.plr_nccl_comm_init(ctypes.byref(h), idbuf, self.rank, self.world), "plr_nccl_comm_init")
         self.handle = h
