@@ -15,9 +15,10 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-# experiment variants: PLR_VARIANT="STAGES,LAG,NL" builds libplr_b200_sS_dD_lNL.so
+# experiment variants: PLR_VARIANT="name:S,D,NL:S,D,NL" (DECAY config, generic
+# config) builds libplr_b200_<name>.so
 _VAR = os.environ.get("PLR_VARIANT")
-_SUFFIX = "" if not _VAR else "_s%s_d%s_l%s" % tuple(_VAR.split(","))
+_SUFFIX = "" if not _VAR else "_" + _VAR.split(":")[0]
 BUILD = os.path.join(HERE, "_build" + _SUFFIX)
 LIB = os.path.join(HERE, "libplr_b200%s.so" % _SUFFIX)
 INCLUDE = os.path.join(os.path.dirname(HERE), "include")
@@ -27,8 +28,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUDE, "-I" + CSRC,
           "--ftz=true", "--prec-div=true", "--prec-sqrt=true", "--fmad=true"]
 if _VAR:
-    COMMON += ["-DPLR_STAGES=%s" % _VAR.split(",")[0], "-DPLR_LAG=%s" % _VAR.split(",")[1],
-               "-DPLR_NL=%s" % _VAR.split(",")[2]]
+    COMMON += ['-DPLR_CFG_DEC=%s' % _VAR.split(":")[1], '-DPLR_CFG_GEN=%s' % _VAR.split(":")[2]]
 
 
 def _sources():

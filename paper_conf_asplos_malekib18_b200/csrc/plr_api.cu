@@ -370,7 +370,7 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->elems_per_thread = plan->pt.geo.X;
     info->threads_per_cta = plan->pt.geo.W * 32;
     info->tile_elems = plan->pt.geo.tile();
-    info->stages = plan->pt.geo.S;
+    info->stages = scan_stages(plan->pt);
     info->decay_len = plan->pt.decay_len;
     info->fixup_len = plan->pt.fixup_len;
     info->n_max = plan->n_max;

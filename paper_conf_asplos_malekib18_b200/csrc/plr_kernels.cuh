@@ -222,7 +222,7 @@ struct Layout {
 };
 
 // ------------------------------------------------------ the scan kernel ----
-template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool STORE>
+template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool DEC, bool STORE>
 __global__ void __launch_bounds__((W + 1 + NL) * 32)
 plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = Layout<T, A, K, X, W, S, D>;
@@ -336,7 +336,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (j == 0) {
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = prm.y_hist != nullptr ? A(prm.y_hist[K - 1 - q]) : A(0);
-            } else if (prm.decay) {
+            } else if (DEC) {
                 // T(m) == 0: every tile published inclusive == aggregate at
                 // once; the look-back is a single hop
                 A v[K];
@@ -465,12 +465,12 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 for (int q = 0; q < K; q++) Gp[q] = acc[q];
             }
             // the tile's own aggregate (phase A) is needed for its inclusive carry
-            if (j == 0 || prm.decay) mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
+            if (j == 0 || DEC) mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
             if (lane == 0) {
 #pragma unroll
                 for (int q = 0; q < K; q++) sG[slot * kMaxK + q] = Gp[q];
             }
-            if (!prm.decay || j == 0) {
+            if (!DEC || j == 0) {
                 A G[K];
 #pragma unroll
                 for (int q = 0; q < K; q++) G[q] = sAt[slot * kMaxK + q];
@@ -583,11 +583,11 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         }
         // publish the tile aggregate at once: "P" for the generic
         // look-back; for DECAY the inclusive carry equals the aggregate
-        if (warp == 0 && (j > 0 || prm.decay)) {
+        if (warp == 0 && (j > 0 || DEC)) {
             A At[K];
 #pragma unroll
             for (int q = 0; q < K; q++) At[q] = shfl_idx(u_[q], W - 1);
-            publish_status<A, K>(prm.status, j, At, prm.decay ? 2u * prm.epoch + 1u : 2u * prm.epoch, lane);
+            publish_status<A, K>(prm.status, j, At, DEC ? 2u * prm.epoch + 1u : 2u * prm.epoch, lane);
         }
         // wagg is buffered per slot: its next writer (tile it+NS) runs after
         // every warp passed tile it+1's barrier
@@ -656,21 +656,18 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         mbar_arrive(&done_bar[s]);
     };
 
-    // software pipeline: phase A runs D tiles ahead of phase B
-    long long jq[NS];
+    // software pipeline: phase A runs D tiles ahead of phase B.  Phase B
+    // reads its tile id from tile_of[], stable until the tile's done barrier.
     int na = 0, nb = 0;                             // phases A / B done
-    for (; na < D; na++) {
-        jq[na % NS] = phaseA(na);
-        if (jq[na % NS] >= ntiles) break;
-    }
+    for (; na < D; na++)
+        if (phaseA(na) >= ntiles) break;
     for (bool stop = na < D; !stop;) {
         const long long j = phaseA(na);
-        jq[na % NS] = j;
-        phaseB(nb, jq[nb % NS]);
+        phaseB(nb, tile_of[nb % S]);
         nb++;
         if (j >= ntiles) stop = true; else na++;
     }
-    for (; nb < na; nb++) phaseB(nb, jq[nb % NS]);   // drain
+    for (; nb < na; nb++) phaseB(nb, tile_of[nb % S]);   // drain
 }
 
 }  // namespace dev

@@ -37,6 +37,9 @@ cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm);
 // per-(data, accumulation) type entry points (plr_scan_*.cu)
 cudaError_t launch_scan_i32(const Tables<uint32_t, uint32_t>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t launch_scan_f32(const Tables<float, float>& tab, const LaunchArgs& la, int k, int p);
-cudaError_t launch_scan_f64acc(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_scan_f64acc_dec(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_scan_f64acc_gen(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
+// ring depth of the config a plan launches with (plan info)
+int scan_stages(const PlanTables& pt);
 
 }  // namespace plr

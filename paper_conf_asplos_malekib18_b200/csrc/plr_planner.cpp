@@ -199,6 +199,7 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         for (int64_t u = 0; u < cap; u++) sg += std::fabs(g[u]);
         pt.cond_bound = std::ldexp(1.0, -24) * sa * sg * sg;
         pt.acc64 = (!decays || !(pt.cond_bound <= 1e-3)) ? 1 : 0;
+        if (!pt.decay_flag) pt.acc64 = 1;      // multi-tile look-back kernels exist in fp64 accumulation only
         if (decays) {
             pt.decay_len = last;
             // free response of the augmented state (x_{-4..-1}, y_{-4..-1})

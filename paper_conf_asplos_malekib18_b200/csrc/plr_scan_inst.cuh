@@ -1,6 +1,6 @@
 // plr_scan_inst.cuh -- host-side launch of the scan kernel for one
-// (data type T, accumulation type A); included by the per-type .cu files so
-// the instantiations compile in parallel.
+// (data type T, accumulation type A, pipeline config); included by the
+// per-type .cu files so the instantiations compile in parallel.
 #pragma once
 #include "plr_kernels.cuh"
 #include "plr_launch.h"
@@ -8,21 +8,35 @@
 namespace plr {
 namespace inst {
 
-#ifndef PLR_STAGES
-#define PLR_STAGES 5
-#endif
-#ifndef PLR_LAG
-#define PLR_LAG 2
-#endif
-#ifndef PLR_NL
-#define PLR_NL 2
-#endif
-constexpr int kX = 15, kW = 8, kS = PLR_STAGES, kD = PLR_LAG, kNL = PLR_NL;   // see default_geometry()
+constexpr int kX = 15, kW = 8;          // m = 3840 (see default_geometry())
 
-template <typename T, typename A, int K, int P, bool STORE>
+// Pipeline configs (measured on B200):
+//   DECAY (single-hop look-back): shallow pipeline, 3 CTAs/SM fit:
+//     S = 4 stages, phase-A lead D = 1, one look-back warp;
+//   generic (multi-tile look-back): deep pipeline so predecessors' aggregates
+//     are published before a tile looks back: S = 6, D = 3, two look-back warps.
+#ifndef PLR_CFG_DEC
+#define PLR_CFG_DEC 4, 1, 1
+#endif
+#ifndef PLR_CFG_GEN
+#define PLR_CFG_GEN 6, 3, 2
+#endif
+
+template <int S_, int D_, int NL_, bool DEC_>
+struct Cfg {
+    static constexpr int S = S_, D = D_, NL = NL_;
+    static constexpr bool DEC = DEC_;
+};
+template <int S_, int D_, int NL_> using DecCfg = Cfg<S_, D_, NL_, true>;
+template <int S_, int D_, int NL_> using GenCfg = Cfg<S_, D_, NL_, false>;
+using CfgDec = DecCfg<PLR_CFG_DEC>;
+using CfgGen = GenCfg<PLR_CFG_GEN>;
+
+template <typename T, typename A, class C, int K, int P, bool STORE>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
-    auto kern = &dev::plr_scan_kernel<T, A, K, P, kX, kW, kS, kD, kNL, STORE>;
-    const size_t smem = dev::Layout<T, A, K, kX, kW, kS, kD>::bytes;
+    auto kern = &dev::plr_scan_kernel<T, A, K, P, kX, kW, C::S, C::D, C::NL, C::DEC, STORE>;
+    const size_t smem = dev::Layout<T, A, K, kX, kW, C::S, C::D>::bytes;
+    constexpr int threads = (kW + 1 + C::NL) * 32;
     static bool configured = false;
     if (!configured) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -30,7 +44,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
         configured = true;
     }
     if (la.occupancy_out != nullptr)    // occupancy query: report CTAs/SM, do not launch
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, (kW + 1 + kNL) * 32, smem);
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, threads, smem);
     ScanParams<T, A> prm;
     prm.x = static_cast<const T*>(la.x);
     prm.y = static_cast<T*>(la.y);
@@ -47,28 +61,28 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     prm.lane_T = static_cast<const A*>(la.lane_T);
     prm.stats = la.stats;
     prm.tab = tab;
-    kern<<<la.grid, (kW + 1 + kNL) * 32, smem, la.stream>>>(prm);
+    kern<<<la.grid, threads, smem, la.stream>>>(prm);
     return cudaGetLastError();
 }
 
-template <typename T, typename A, int K>
+template <typename T, typename A, class C, int K>
 cudaError_t launch_k(const Tables<T, A>& tab, const LaunchArgs& la, int p) {
     switch (p) {
-        case 0: return la.store ? launch_kps<T, A, K, 0, true>(tab, la) : launch_kps<T, A, K, 0, false>(tab, la);
-        case 1: return la.store ? launch_kps<T, A, K, 1, true>(tab, la) : launch_kps<T, A, K, 1, false>(tab, la);
-        case 2: return la.store ? launch_kps<T, A, K, 2, true>(tab, la) : launch_kps<T, A, K, 2, false>(tab, la);
-        case 3: return la.store ? launch_kps<T, A, K, 3, true>(tab, la) : launch_kps<T, A, K, 3, false>(tab, la);
+        case 0: return la.store ? launch_kps<T, A, C, K, 0, true>(tab, la) : launch_kps<T, A, C, K, 0, false>(tab, la);
+        case 1: return la.store ? launch_kps<T, A, C, K, 1, true>(tab, la) : launch_kps<T, A, C, K, 1, false>(tab, la);
+        case 2: return la.store ? launch_kps<T, A, C, K, 2, true>(tab, la) : launch_kps<T, A, C, K, 2, false>(tab, la);
+        case 3: return la.store ? launch_kps<T, A, C, K, 3, true>(tab, la) : launch_kps<T, A, C, K, 3, false>(tab, la);
     }
     return cudaErrorInvalidValue;
 }
 
-template <typename T, typename A>
+template <typename T, typename A, class C>
 cudaError_t launch(const Tables<T, A>& tab, const LaunchArgs& la, int k, int p) {
     switch (k) {
-        case 1: return launch_k<T, A, 1>(tab, la, p);
-        case 2: return launch_k<T, A, 2>(tab, la, p);
-        case 3: return launch_k<T, A, 3>(tab, la, p);
-        case 4: return launch_k<T, A, 4>(tab, la, p);
+        case 1: return launch_k<T, A, C, 1>(tab, la, p);
+        case 2: return launch_k<T, A, C, 2>(tab, la, p);
+        case 3: return launch_k<T, A, C, 3>(tab, la, p);
+        case 4: return launch_k<T, A, C, 4>(tab, la, p);
     }
     return cudaErrorInvalidValue;
 }
