@@ -116,8 +116,10 @@ plr_status plr_plan_factor_lists(const plr_plan* plan, int64_t m, void* out);
 
 /* Debug counters of the generic look-back, enabled by PLR_STATS=1 in the
  * environment at plan creation (otherwise all zero): out[0] look-backs,
- * out[1] windows read, out[2] waits on a not-ready tile, out[3] summed
- * depth in tiles.  Synchronous; reset != 0 clears them.  Host memory. */
+ * out[1] window polls, out[2] polls that folded nothing, out[3] summed
+ * depth in tiles, out[4] SM cycles waiting for the tile's own aggregate,
+ * out[5] cycles looking back, out[6] of which sleeping.  Synchronous;
+ * reset != 0 clears them.  Host memory. */
 plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out /* 8 */, int reset);
 
 /* y[0..n) = recurrence over x[0..n) with zero initial conditions.

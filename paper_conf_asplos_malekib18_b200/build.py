@@ -15,8 +15,8 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-# experiment variants: PLR_VARIANT="name:S,D,NL:S,D,NL" (DECAY config, generic
-# config) builds libplr_b200_<name>.so
+# experiment variants: PLR_VARIANT="name:S.D.NL:S.D.NL[:DEFS]" (DECAY config,
+# generic config, extra defines joined by '+') builds libplr_b200_<name>.so
 _VAR = os.environ.get("PLR_VARIANT")
 _SUFFIX = "" if not _VAR else "_" + _VAR.split(":")[0]
 BUILD = os.path.join(HERE, "_build" + _SUFFIX)
@@ -27,8 +27,13 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUDE, "-I" + CSRC,
           "--ftz=true", "--prec-div=true", "--prec-sqrt=true", "--fmad=true"]
-if _VAR:
-    COMMON += ['-DPLR_CFG_DEC=%s' % _VAR.split(":")[1], '-DPLR_CFG_GEN=%s' % _VAR.split(":")[2]]
+if _VAR:   # name:S.D.NL:S.D.NL[:extra -D defines separated by +]  (nvcc splits -D values on ',')
+    _p = _VAR.split(":")
+    for _tag, _cfg in (("DEC", _p[1]), ("GEN", _p[2])):
+        _s, _d, _l = _cfg.split(".")
+        COMMON += ["-DPLR_%s_S=%s" % (_tag, _s), "-DPLR_%s_D=%s" % (_tag, _d), "-DPLR_%s_NL=%s" % (_tag, _l)]
+    if len(_p) > 3:
+        COMMON += ["-D" + d for d in _p[3].split("+") if d]
 
 
 def _sources():

@@ -358,7 +358,10 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 // and never re-reads folded tiles.  Start once the tile's own
                 // aggregate is published: the predecessors of the same wave
                 // have had the same time to publish theirs.
+                const long long c_start = clock64();
                 mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
+                const long long c_agg = clock64();
+                long long c_wait = 0;
                 A acc[K];
                 A Tacc[K * kMaxK];
 #pragma unroll
@@ -368,8 +371,14 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     for (int r = 0; r < kMaxK; r++) Tacc[q * kMaxK + r] = (q == r) ? A(1) : A(0);
                 }
                 long long o = 0;                   // distance of the first unfolded tile from j-1
-                int ltpl = 1;                      // log2 tiles per lane: 2 (64-tile window), then 8
-                int ns = 32;
+#ifndef PLR_LB_LTPL0
+#define PLR_LB_LTPL0 1
+#endif
+                int ltpl = PLR_LB_LTPL0;           // log2 tiles per lane: 2 (64-tile window), then 8
+#ifndef PLR_LB_NS0
+#define PLR_LB_NS0 32
+#endif
+                int ns = PLR_LB_NS0;
                 unsigned long long n_win = 0, n_wait = 0;
                 for (;;) {
                     n_win++;
@@ -447,11 +456,13 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                                 for (int c2 = 0; c2 < K; c2++) Tacc[q * kMaxK + c2] = nt[q * kMaxK + c2];
                         }
                         o += e;
-                        ns = 32;
+                        ns = PLR_LB_NS0;
                         if (!bn) ltpl = 3;                         // nothing pending: widen to 256 tiles
                     } else {
                         n_wait++;                                  // nearest tile not ready yet
+                        const long long cw = clock64();
                         __nanosleep(ns);
+                        c_wait += clock64() - cw;
                         ns = ns < 512 ? 2 * ns : ns;
                     }
                 }
@@ -460,6 +471,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     atomicAdd(&prm.stats[1], n_win);               // window polls
                     atomicAdd(&prm.stats[2], n_wait);              // polls that folded nothing
                     atomicAdd(&prm.stats[3], (unsigned long long)(o + 1));  // depth folded (approx.)
+                    atomicAdd(&prm.stats[4], (unsigned long long)(c_agg - c_start));    // cycles waiting own A
+                    atomicAdd(&prm.stats[5], (unsigned long long)(clock64() - c_agg));  // cycles looking back
+                    atomicAdd(&prm.stats[6], (unsigned long long)c_wait);               // of which sleeping
                 }
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = acc[q];

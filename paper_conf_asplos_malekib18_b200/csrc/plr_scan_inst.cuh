@@ -15,11 +15,15 @@ constexpr int kX = 15, kW = 8;          // m = 3840 (see default_geometry())
 //     S = 4 stages, phase-A lead D = 1, one look-back warp;
 //   generic (multi-tile look-back): deep pipeline so predecessors' aggregates
 //     are published before a tile looks back: S = 6, D = 3, two look-back warps.
-#ifndef PLR_CFG_DEC
-#define PLR_CFG_DEC 4, 1, 1
+#ifndef PLR_DEC_S
+#define PLR_DEC_S 4
+#define PLR_DEC_D 1
+#define PLR_DEC_NL 1
 #endif
-#ifndef PLR_CFG_GEN
-#define PLR_CFG_GEN 6, 3, 2
+#ifndef PLR_GEN_S
+#define PLR_GEN_S 6
+#define PLR_GEN_D 3
+#define PLR_GEN_NL 2
 #endif
 
 template <int S_, int D_, int NL_, bool DEC_>
@@ -29,8 +33,8 @@ struct Cfg {
 };
 template <int S_, int D_, int NL_> using DecCfg = Cfg<S_, D_, NL_, true>;
 template <int S_, int D_, int NL_> using GenCfg = Cfg<S_, D_, NL_, false>;
-using CfgDec = DecCfg<PLR_CFG_DEC>;
-using CfgGen = GenCfg<PLR_CFG_GEN>;
+using CfgDec = DecCfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL>;
+using CfgGen = GenCfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL>;
 
 template <typename T, typename A, class C, int K, int P, bool STORE>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
