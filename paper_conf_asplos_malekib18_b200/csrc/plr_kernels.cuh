@@ -222,8 +222,11 @@ struct Layout {
 };
 
 // ------------------------------------------------------ the scan kernel ----
+#ifndef PLR_MIN_CTAS
+#define PLR_MIN_CTAS 1
+#endif
 template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool DEC, bool STORE>
-__global__ void __launch_bounds__((W + 1 + NL) * 32)
+__global__ void __launch_bounds__((W + 1 + NL) * 32, PLR_MIN_CTAS)
 plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = Layout<T, A, K, X, W, S, D>;
     constexpr int NS = L::NS;
@@ -360,6 +363,16 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 // have had the same time to publish theirs.
                 const long long c_start = clock64();
                 mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
+#ifndef PLR_LB_START
+#define PLR_LB_START 0
+#endif
+                if (PLR_LB_START > 0 && D > 1) {
+                    // start one tile later: the CTA's next aggregate is published,
+                    // so are most predecessors' (phase B of this tile is still
+                    // D-1 tiles away)
+                    const int nx = it + 1;
+                    mbar_wait(&agg_bar[nx % NS], (uint32_t)((nx / NS) & 1));
+                }
                 const long long c_agg = clock64();
                 long long c_wait = 0;
                 A acc[K];

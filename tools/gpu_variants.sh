@@ -1,6 +1,6 @@
 set -x
 rm -f gpurun_out/lbstats.log
-for v in "" _w3 _ns0 _l4; do
+for v in _lb4 _lb4s _s2; do
   echo "== variant '$v'" >> gpurun_out/lbstats.log
-  PLR_LIB=$PWD/paper_conf_asplos_malekib18_b200/libplr_b200$v.so timeout 300 python tools/lookback_stats.py $((1<<30)) prefix,tuple2,tuple3,lp1 >> gpurun_out/lbstats.log 2>&1
+  PLR_LIB=$PWD/paper_conf_asplos_malekib18_b200/libplr_b200$v.so timeout 300 python tools/lookback_stats.py $((1<<30)) prefix,tuple2,tuple3,order3 >> gpurun_out/lbstats.log 2>&1
 done
