@@ -165,31 +165,52 @@ template <> struct StatusIO<double> {
     }
 };
 
-// publish carry vector `val` of tile j with `tag`; lanes 0..K*kWords-1 of the
-// calling warp each store one 64-bit word
+// Status records are packed at a power-of-two stride of NW 64-bit words per
+// tile (NW = K words for 32-bit carries, 2K for fp64), so a window of
+// consecutive tiles is one contiguous block and a warp-wide load of 32
+// consecutive tiles coalesces into a few L2 requests.
+template <typename A, int K>
+struct StatusLayout {
+    static constexpr int NW = K * StatusIO<A>::kWords;
+    static constexpr int STRIDE = NW <= 1 ? 1 : NW <= 2 ? 2 : NW <= 4 ? 4 : 8;
+};
+
+__device__ __forceinline__ void ld_relaxed_v2(const unsigned long long* p, unsigned long long& a,
+                                              unsigned long long& b) {
+    asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+
+// publish carry vector `val` of tile j with `tag`; lanes 0..NW-1 of the
+// calling warp each store one 64-bit word (single-copy atomic per word)
 template <typename A, int K>
 __device__ __forceinline__ void publish_status(unsigned long long* status, long long j, const A (&val)[K],
                                                uint32_t tag, int lane) {
     using SIO = StatusIO<A>;
-    constexpr int NW = K * SIO::kWords;
-    unsigned long long* stj = status + (size_t)j * (2 * kStatusWords);
-    unsigned long long w[NW];
+    using SL = StatusLayout<A, K>;
+    unsigned long long* stj = status + (size_t)j * SL::STRIDE;
+    unsigned long long w[SL::NW];
 #pragma unroll
     for (int q = 0; q < K; q++) SIO::pack(val[q], tag, &w[q * SIO::kWords]);
 #pragma unroll
-    for (int e = 0; e < NW; e++) if (lane == e) st_relaxed(stj + e, w[e]);
+    for (int e = 0; e < SL::NW; e++) if (lane == e) st_relaxed(stj + e, w[e]);
 }
 
-// read tile jj's K components: 2 inclusive, 1 aggregate, 0 not ready
+// read tile jj's K components: 2 inclusive, 1 aggregate, 0 not ready.  Every
+// word carries its own tag, so 16-byte vector loads (two relaxed 64-bit
+// accesses) are as safe as scalar ones.
 template <typename A, int K>
 __device__ __forceinline__ int read_status(const unsigned long long* status, long long jj, A (&val)[K],
                                            uint32_t tagA, uint32_t tagI) {
     using SIO = StatusIO<A>;
-    constexpr int NW = K * SIO::kWords;
-    const unsigned long long* sp = status + (size_t)jj * (2 * kStatusWords);
-    unsigned long long w[NW];
+    using SL = StatusLayout<A, K>;
+    constexpr int NW = SL::NW;
+    const unsigned long long* sp = status + (size_t)jj * SL::STRIDE;
+    unsigned long long w[NW + 1];
 #pragma unroll
-    for (int e = 0; e < NW; e++) w[e] = ld_relaxed(sp + e);
+    for (int e = 0; e + 1 < NW + (NW & 1); e += 2) {
+        if (e + 1 < NW) ld_relaxed_v2(sp + e, w[e], w[e + 1]);
+        else w[e] = ld_relaxed(sp + e);
+    }
     bool allI = true, allA = true;
 #pragma unroll
     for (int q = 0; q < K; q++) {
@@ -396,6 +417,8 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 for (;;) {
                     n_win++;
                     const int tpl = 1 << ltpl;
+                    // lane-interleaved window: distance d = o + 32 t + lane, t < tpl,
+                    // so every warp-wide load reads 32 consecutive tiles
                     A v[kTPL][K];
                     int st[kTPL];
 #pragma unroll
@@ -404,45 +427,43 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
                         for (int q = 0; q < K; q++) v[t][q] = A(0);
                         if (t < tpl) {
-                            const long long jj = j - 1 - (o + (long long)lane * tpl + t);
+                            const long long jj = j - 1 - (o + 32LL * t + lane);
                             if (jj >= 0) st[t] = read_status<A, K>(prm.status, jj, v[t], tagA, tagI);
                         }
                     }
-                    int fi = kTPL, fn = kTPL;                    // first inclusive / not-ready in lane
+                    int di = 1 << 30, dn = 1 << 30;              // lane's nearest inclusive / not-ready
 #pragma unroll
                     for (int t = kTPL - 1; t >= 0; t--) {
-                        if (t < tpl && st[t] == 2) fi = t;
-                        if (t < tpl && st[t] == 0) fn = t;
+                        if (t < tpl && st[t] == 2) di = 32 * t + lane;
+                        if (t < tpl && st[t] == 0) dn = 32 * t + lane;
                     }
-                    const unsigned bi = __ballot_sync(0xffffffffu, fi < tpl);
-                    const unsigned bn = __ballot_sync(0xffffffffu, fn < tpl);
-                    const int dI = bi ? (__ffs(bi) - 1) * tpl + shfl_idx(fi, __ffs(bi) - 1) : 1 << 30;
-                    const int dN = bn ? (__ffs(bn) - 1) * tpl + shfl_idx(fn, __ffs(bn) - 1) : 1 << 30;
+                    const int dI = __reduce_min_sync(0xffffffffu, (unsigned)di);
+                    const int dN = __reduce_min_sync(0xffffffffu, (unsigned)dn);
                     const bool found = dI < dN;
-                    const int e = found ? dI + 1 : (bn ? dN : 32 * tpl);   // tiles to fold now
+                    const int e = found ? dI + 1 : (dN < (1 << 30) ? dN : 32 * tpl);   // tiles to fold now
                     if (e > 0) {
-                        // per-lane Horner over its tiles with window offset < e
+                        // per-lane Horner over t (stride 32 tiles), then a tree over lanes
                         A r[K];
 #pragma unroll
                         for (int q = 0; q < K; q++) r[q] = A(0);
 #pragma unroll
                         for (int t = kTPL - 1; t >= 0; t--) {
-                            if (t < tpl && lane * tpl + t < e) {
+                            if (t < tpl && 32 * t + lane < e) {
                                 A nr[K];
 #pragma unroll
                                 for (int q = 0; q < K; q++) nr[q] = v[t][q];
-                                matvec_acc<A, K>(nr, tb.Tm, r);
+                                matvec_acc<A, K>(nr, tb.Tpow[5], r);           // T(32 m)
 #pragma unroll
                                 for (int q = 0; q < K; q++) r[q] = nr[q];
                             }
                         }
-                        // tree over lanes: R = sum_l T(l tpl m) r_l, T(tpl m 2^s) = Tpow[ltpl + s]
+                        // R = sum_l T(l m) r_l, T(m 2^s) = Tpow[s]
 #pragma unroll
                         for (int s2 = 0; s2 < 5; s2++) {
                             A o2[K];
 #pragma unroll
                             for (int q = 0; q < K; q++) o2[q] = shfl_down(r[q], 1 << s2);
-                            matvec_acc<A, K>(r, tb.Tpow[ltpl + s2], o2);
+                            matvec_acc<A, K>(r, tb.Tpow[s2], o2);
                         }
                         A R[K];
 #pragma unroll
@@ -470,7 +491,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                         }
                         o += e;
                         ns = PLR_LB_NS0;
-                        if (!bn) ltpl = 3;                         // nothing pending: widen to 256 tiles
+                        if (dN >= (1 << 30)) ltpl = 3;             // nothing pending: widen to 256 tiles
                     } else {
                         n_wait++;                                  // nearest tile not ready yet
                         const long long cw = clock64();
