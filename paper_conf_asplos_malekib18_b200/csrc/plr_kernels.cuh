@@ -169,10 +169,15 @@ template <> struct StatusIO<double> {
 // tile (NW = K words for 32-bit carries, 2K for fp64), so a window of
 // consecutive tiles is one contiguous block and a warp-wide load of 32
 // consecutive tiles coalesces into a few L2 requests.
+#ifndef PLR_STATUS_MIN_STRIDE
+#define PLR_STATUS_MIN_STRIDE 4
+#endif
 template <typename A, int K>
 struct StatusLayout {
     static constexpr int NW = K * StatusIO<A>::kWords;
-    static constexpr int STRIDE = NW <= 1 ? 1 : NW <= 2 ? 2 : NW <= 4 ? 4 : 8;
+    static constexpr int P2 = NW <= 1 ? 1 : NW <= 2 ? 2 : NW <= 4 ? 4 : 8;
+    static constexpr int STRIDE = P2 > PLR_STATUS_MIN_STRIDE ? P2 : PLR_STATUS_MIN_STRIDE;
+    static_assert(STRIDE * 8 <= kStatusMaxBytes, "status record stride");
 };
 
 __device__ __forceinline__ void ld_relaxed_v2(const unsigned long long* p, unsigned long long& a,
