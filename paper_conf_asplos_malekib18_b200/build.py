@@ -15,7 +15,7 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-# experiment variants: PLR_VARIANT="name:S.D.NL:S.D.NL[:DEFS]" (DECAY config,
+# experiment variants: PLR_VARIANT="name:S.D.NL[.X.W]:S.D.NL[.X.W][:DEFS]" (DECAY config,
 # generic config, extra defines joined by '+') builds libplr_b200_<name>.so
 _VAR = os.environ.get("PLR_VARIANT")
 _SUFFIX = "" if not _VAR else "_" + _VAR.split(":")[0]
@@ -30,8 +30,9 @@ COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUD
 if _VAR:   # name:S.D.NL:S.D.NL[:extra -D defines separated by +]  (nvcc splits -D values on ',')
     _p = _VAR.split(":")
     for _tag, _cfg in (("DEC", _p[1]), ("GEN", _p[2])):
-        _s, _d, _l = _cfg.split(".")
-        COMMON += ["-DPLR_%s_S=%s" % (_tag, _s), "-DPLR_%s_D=%s" % (_tag, _d), "-DPLR_%s_NL=%s" % (_tag, _l)]
+        _v = _cfg.split(".") + ["15", "8"][len(_cfg.split(".")) - 3:]
+        for _name, _val in zip(("S", "D", "NL", "X", "W"), _v):
+            COMMON += ["-DPLR_%s_%s=%s" % (_tag, _name, _val)]
     if len(_p) > 3:
         COMMON += ["-D" + d for d in _p[3].split("+") if d]
 

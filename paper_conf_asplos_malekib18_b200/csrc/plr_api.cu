@@ -310,7 +310,13 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     *out = nullptr;
     plr_plan* plan = new plr_plan();
     const char* why = "";
-    plr_status st = plan_tables(a, p, b, k, dtype, default_geometry(dtype, k, p), &plan->pt, &why);
+    // plan with the DECAY geometry; non-decaying plans are re-planned with
+    // the generic kernel's geometry (the class is known after planning)
+    plr_status st = plan_tables(a, p, b, k, dtype, class_geometry(true), &plan->pt, &why);
+    if (st == PLR_OK && !plan->pt.decay_flag) {
+        plan_tables_free(&plan->pt);
+        st = plan_tables(a, p, b, k, dtype, class_geometry(false), &plan->pt, &why);
+    }
     if (st != PLR_OK) {
         delete plan;
         return fail(st, why);

@@ -3,11 +3,11 @@
 
 namespace plr {
 
-Geometry default_geometry(plr_dtype, int, int) {
-    // x = 15 elements per thread (odd: conflict-free strided smem access),
-    // 8 compute warps: m = 3840 elements = 15 KB per tile.  The ring depth
-    // depends on the class (scan_stages()).
-    return Geometry{inst::kX, inst::kW, 0};
+Geometry class_geometry(bool decay) {
+    // x elements per thread (odd: conflict-free strided smem access) and W
+    // compute warps per config; the ring depth is reported by scan_stages()
+    return decay ? Geometry{inst::CfgDec::X, inst::CfgDec::W, inst::CfgDec::S}
+                 : Geometry{inst::CfgGen::X, inst::CfgGen::W, inst::CfgGen::S};
 }
 
 int scan_stages(const PlanTables& pt) {

@@ -28,8 +28,8 @@ struct LaunchArgs {
     int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel
 };
 
-// Tile geometry per dtype/order (must match an instantiated kernel).
-Geometry default_geometry(plr_dtype dtype, int k, int p);
+// Tile geometry of the DECAY / generic kernel configs.
+Geometry class_geometry(bool decay);
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm);

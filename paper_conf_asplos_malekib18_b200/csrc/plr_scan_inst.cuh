@@ -8,8 +8,6 @@
 namespace plr {
 namespace inst {
 
-constexpr int kX = 15, kW = 8;          // m = 3840 (see default_geometry())
-
 // Pipeline configs (measured on B200):
 //   DECAY (single-hop look-back): shallow pipeline, 3 CTAs/SM fit:
 //     S = 4 stages, phase-A lead D = 1, one look-back warp;
@@ -19,28 +17,32 @@ constexpr int kX = 15, kW = 8;          // m = 3840 (see default_geometry())
 #define PLR_DEC_S 4
 #define PLR_DEC_D 1
 #define PLR_DEC_NL 1
+#define PLR_DEC_X 15
+#define PLR_DEC_W 8
 #endif
 #ifndef PLR_GEN_S
 #define PLR_GEN_S 6
 #define PLR_GEN_D 3
 #define PLR_GEN_NL 2
+#define PLR_GEN_X 15
+#define PLR_GEN_W 8
 #endif
 
-template <int S_, int D_, int NL_, bool DEC_>
+// S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
+// W compute warps (tile m = 32 W X)
+template <int S_, int D_, int NL_, int X_, int W_, bool DEC_>
 struct Cfg {
-    static constexpr int S = S_, D = D_, NL = NL_;
+    static constexpr int S = S_, D = D_, NL = NL_, X = X_, W = W_;
     static constexpr bool DEC = DEC_;
 };
-template <int S_, int D_, int NL_> using DecCfg = Cfg<S_, D_, NL_, true>;
-template <int S_, int D_, int NL_> using GenCfg = Cfg<S_, D_, NL_, false>;
-using CfgDec = DecCfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL>;
-using CfgGen = GenCfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL>;
+using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, true>;
+using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, false>;
 
 template <typename T, typename A, class C, int K, int P, bool STORE>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
-    auto kern = &dev::plr_scan_kernel<T, A, K, P, kX, kW, C::S, C::D, C::NL, C::DEC, STORE>;
-    const size_t smem = dev::Layout<T, A, K, kX, kW, C::S, C::D>::bytes;
-    constexpr int threads = (kW + 1 + C::NL) * 32;
+    auto kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE>;
+    const size_t smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
+    constexpr int threads = (C::W + 1 + C::NL) * 32;
     static bool configured = false;
     if (!configured) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

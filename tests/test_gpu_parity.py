@@ -12,7 +12,7 @@ import workloads
 pytestmark = pytest.mark.gpu
 
 TOL = 1e-4
-M = 3840                 # tile of the default geometry (checked below)
+M = 3840                 # nominal tile (DECAY kernels); sizes below span many tiles either way
 
 
 def rel_err(y, ref):
@@ -38,15 +38,18 @@ def run(plr, torch, sig, x, n_max=None):
     return y
 
 
-SIZES = [1, 2, 3, 4, 5, 14, 15, 16, 31, 32, 33, 480, 481, M - 1, M, M + 1, 3 * M + 7, 33 * M + 5,
-         (1 << 16) + 3, (1 << 20) + 12345]
+def sizes_for(m):
+    """Edge sizes around the plan's tile m (the generic and DECAY kernels use
+    different tiles), several tiles with ragged tails, and larger sizes."""
+    return [1, 2, 3, 4, 5, 14, 15, 16, 31, 32, 33, 480, 481, m - 1, m, m + 1, 3 * m + 7, 33 * m + 5,
+            (1 << 16) + 3, (1 << 20) + 12345]
 
 
 @pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
 def test_parity_sizes(cuda_plr, sig):
     import torch
-    info = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 10).info
-    assert info["tile_elems"] == M
+    m = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 10).info["tile_elems"]
+    SIZES = sizes_for(m)
     x_all = workloads.host_input(max(SIZES), sig.dtype, workloads.seed_for(1))
     plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=max(SIZES))
     for n in SIZES:
