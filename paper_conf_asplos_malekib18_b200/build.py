@@ -30,8 +30,8 @@ COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUD
 if _VAR:   # name:S.D.NL:S.D.NL[:extra -D defines separated by +]  (nvcc splits -D values on ',')
     _p = _VAR.split(":")
     for _tag, _cfg in (("DEC", _p[1]), ("GEN", _p[2])):
-        _v = _cfg.split(".") + ["15", "8"][len(_cfg.split(".")) - 3:]
-        for _name, _val in zip(("S", "D", "NL", "X", "W"), _v):
+        _v = _cfg.split(".") + ["15", "8", "3" if _tag == "DEC" else "2"][len(_cfg.split(".")) - 3:]
+        for _name, _val in zip(("S", "D", "NL", "X", "W", "MINB"), _v):
             COMMON += ["-DPLR_%s_%s=%s" % (_tag, _name, _val)]
     if len(_p) > 3:
         COMMON += ["-D" + d for d in _p[3].split("+") if d]

@@ -248,11 +248,9 @@ struct Layout {
 };
 
 // ------------------------------------------------------ the scan kernel ----
-#ifndef PLR_MIN_CTAS
-#define PLR_MIN_CTAS 1
-#endif
-template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool DEC, bool STORE>
-__global__ void __launch_bounds__((W + 1 + NL) * 32, PLR_MIN_CTAS)
+template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool DEC, bool STORE,
+          int MINB>
+__global__ void __launch_bounds__((W + 1 + NL) * 32, MINB)
 plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = Layout<T, A, K, X, W, S, D>;
     constexpr int NS = L::NS;
@@ -577,7 +575,13 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             }
         }
         // a2: sequential local recurrence with zero state, in A
-        A l[X];
+        // chunk values are kept in the data type (phase B corrects them);
+        // only the last K live in the accumulation type.  The oldest term is
+        // added first so the newest value l_{u-1} is on the critical path once.
+        T lf[X];
+        A hist[K];                                              // hist[r-1] = l_{u-r}
+#pragma unroll
+        for (int r = 0; r < K; r++) hist[r] = A(0);
 #pragma unroll
         for (int u = 0; u < X; u++) {
             T t = tb.alpha[0] * xv[P + u];
@@ -585,13 +589,16 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             for (int q = 1; q <= P; q++) t = mad(tb.alpha[q], xv[P + u - q], t);
             A acc = A(t);
 #pragma unroll
-            for (int r = 1; r <= K; r++)
-                if (u - r >= 0) acc = mad(tb.c[r - 1], l[u - r], acc);
-            l[u] = acc;
+            for (int r = K; r >= 1; r--)
+                if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
+#pragma unroll
+            for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
+            hist[0] = acc;
+            lf[u] = T(acc);
         }
         A v[K];
 #pragma unroll
-        for (int q = 0; q < K; q++) v[q] = l[X - 1 - q];       // local carry (l_{X-1}, ..., l_{X-K})
+        for (int q = 0; q < K; q++) v[q] = hist[q];             // local carry (l_{X-1}, ..., l_{X-K})
 
         // a3: warp inclusive scan with T(X * 2^s)
 #pragma unroll
@@ -614,7 +621,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 
         // keep the chunk values for phase B in place of x (data type)
 #pragma unroll
-        for (int u = 0; u < X; u++) st[kHalo + tid * X + u] = T(l[u]);
+        for (int u = 0; u < X; u++) st[kHalo + tid * X + u] = lf[u];
 
         // a4: scan of the W warp aggregates with T(32X * 2^s)
         A u_[K];

@@ -19,6 +19,7 @@ namespace inst {
 #define PLR_DEC_NL 1
 #define PLR_DEC_X 15
 #define PLR_DEC_W 8
+#define PLR_DEC_MINB 3
 #endif
 #ifndef PLR_GEN_S
 #define PLR_GEN_S 6
@@ -26,21 +27,23 @@ namespace inst {
 #define PLR_GEN_NL 2
 #define PLR_GEN_X 15
 #define PLR_GEN_W 8
+#define PLR_GEN_MINB 2
 #endif
 
 // S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
 // W compute warps (tile m = 32 W X)
-template <int S_, int D_, int NL_, int X_, int W_, bool DEC_>
+// W compute warps (tile m = 32 W X); MINB: CTAs per SM the registers must allow
+template <int S_, int D_, int NL_, int X_, int W_, int MINB_, bool DEC_>
 struct Cfg {
-    static constexpr int S = S_, D = D_, NL = NL_, X = X_, W = W_;
+    static constexpr int S = S_, D = D_, NL = NL_, X = X_, W = W_, MINB = MINB_;
     static constexpr bool DEC = DEC_;
 };
-using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, true>;
-using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, false>;
+using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true>;
+using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false>;
 
 template <typename T, typename A, class C, int K, int P, bool STORE>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
-    auto kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE>;
+    auto kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB>;
     const size_t smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
     constexpr int threads = (C::W + 1 + C::NL) * 32;
     static bool configured = false;

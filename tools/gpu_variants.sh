@@ -1,7 +1,6 @@
 set -x
 rm -f gpurun_out/lbstats.log
-for v in "" _b16l4 _b16l2 _x31l4; do
+for v in "" _g1 _g2 _g3 _g4; do
   echo "== variant '$v'" >> gpurun_out/lbstats.log
-  PLR_LIB=$PWD/paper_conf_asplos_malekib18_b200/libplr_b200$v.so timeout 300 python tools/lookback_stats.py $((1<<30)) prefix,tuple2,tuple3,order3 >> gpurun_out/lbstats.log 2>&1
+  PLR_LIB=$PWD/paper_conf_asplos_malekib18_b200/libplr_b200$v.so timeout 300 python tools/lookback_stats.py $((1<<30)) prefix,tuple2,tuple3,order3,lp1,lp3,hp3 >> gpurun_out/lbstats.log 2>&1
 done
-PLR_LIB=$PWD/paper_conf_asplos_malekib18_b200/libplr_b200_b16l4.so timeout 300 python -m pytest tests/test_gpu_parity.py -x -q -k "not full_size and not host_pipeline" > gpurun_out/pytest_quick.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_quick.log
