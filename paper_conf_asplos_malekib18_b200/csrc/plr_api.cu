@@ -39,6 +39,7 @@ struct plr_plan {
     int ctas_per_sm = 0;
     size_t n_max = 0;
     uint64_t max_tiles = 0;
+    uint64_t status_slots = 0;              // power of two >= max_tiles
     unsigned long long* d_ticket = nullptr;
     unsigned long long ticket_base = 0;
     unsigned long long* d_status = nullptr;
@@ -213,7 +214,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     const uint64_t m = (uint64_t)plan->pt.geo.tile();
     const uint64_t ntiles = (n + m - 1) / m;
     if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
-        CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->max_tiles * kStatusMaxBytes, stream), "status reset");
+        CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, stream), "status reset");
         CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, 8, stream), "ticket reset");
         plan->epoch = 0;
         plan->ticket_base = 0;
@@ -226,6 +227,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.ticket_base = plan->ticket_base;
     la.ticket = plan->d_ticket;
     la.status = plan->d_status;
+    la.status_mask = plan->status_slots - 1;
     la.epoch = plan->epoch;
     la.decay = plan->pt.decay_flag;
     la.x_hist = x_hist; la.y_hist = y_hist; la.y_tail = y_tail;
@@ -341,10 +343,13 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     if (plan->ctas_per_sm < 1) { plr_plan_destroy(plan); return fail(PLR_ERR_CUDA, "kernel does not fit on an SM"); }
     const uint64_t m = (uint64_t)plan->pt.geo.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
+    if (plan->max_tiles > (1ull << 31)) { plr_plan_destroy(plan); return fail(PLR_ERR_SIZE, "n_max too large"); }
+    plan->status_slots = 1;
+    while (plan->status_slots < plan->max_tiles) plan->status_slots <<= 1;
     if ((e = cudaMalloc(&plan->d_ticket, 8)) != cudaSuccess) return bail(e, "alloc ticket");
-    if ((e = cudaMalloc(&plan->d_status, plan->max_tiles * kStatusMaxBytes)) != cudaSuccess) return bail(e, "alloc status");
+    if ((e = cudaMalloc(&plan->d_status, plan->status_slots * kStatusMaxBytes)) != cudaSuccess) return bail(e, "alloc status");
     if ((e = cudaMemset(plan->d_ticket, 0, 8)) != cudaSuccess) return bail(e, "memset");
-    if ((e = cudaMemset(plan->d_status, 0, plan->max_tiles * kStatusMaxBytes)) != cudaSuccess) return bail(e, "memset");
+    if ((e = cudaMemset(plan->d_status, 0, plan->status_slots * kStatusMaxBytes)) != cudaSuccess) return bail(e, "memset");
     const bool acc64 = dtype == PLR_FLOAT32 && plan->pt.acc64;
     const size_t lane_bytes = (size_t)k * k * 32 * (acc64 ? 8 : 4);
     if ((e = cudaMalloc(&plan->d_lane, lane_bytes)) != cudaSuccess) return bail(e, "alloc lane table");
@@ -380,7 +385,7 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->decay_len = plan->pt.decay_len;
     info->fixup_len = plan->pt.fixup_len;
     info->n_max = plan->n_max;
-    info->scratch_bytes = 8 + plan->max_tiles * kStatusMaxBytes + (size_t)plan->pt.k * plan->pt.k * 128 +
+    info->scratch_bytes = 8 + plan->status_slots * kStatusMaxBytes + (size_t)plan->pt.k * plan->pt.k * 128 +
                           (size_t)plan->pt.fixup_len * kAug * 4 + 64;
     info->ctas_per_sm = plan->ctas_per_sm;
     info->num_sms = plan->num_sms;

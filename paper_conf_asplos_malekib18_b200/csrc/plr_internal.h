@@ -18,7 +18,7 @@ constexpr int kHalo = 4;            // words in front of each stage: x_{-4}..x_{
 constexpr int kMaxX = 31;
 constexpr int kMaxW = 16;
 constexpr int kStatusWords = 4;     // u64 status words per tile (>= kMaxK)
-constexpr int kStatusMaxBytes = 128; // status bytes per tile the plan allocates (max record stride)
+constexpr int kStatusMaxBytes = 64;  // bytes per status slot the plan allocates (max record stride)
 constexpr int kAug = 8;             // augmented state slots: x_{-4..-1}, y_{-4..-1}
 constexpr int kTPL = 8;             // look-back: tiles per lane in a wide window (2^3)
 
@@ -53,7 +53,8 @@ struct ScanParams {
     uint64_t ntiles;
     unsigned long long ticket_base;
     unsigned long long* ticket;
-    unsigned long long* status;          // ntiles x kStatusWords, {tag:32 | value:32}
+    unsigned long long* status;          // 2^c scattered records of {tag:32 | value:32} words
+    uint32_t status_mask;                // 2^c - 1, 2^c >= ntiles
     uint32_t epoch;                      // tags 2*epoch (aggregate) / 2*epoch+1 (inclusive)
     int decay;                           // T(m) == 0 exactly: inclusive == aggregate
     const T* x_hist;                     // p values x_{-p}..x_{-1} or null

@@ -169,24 +169,24 @@ template <> struct StatusIO<double> {
 // tile (NW = K words for 32-bit carries, 2K for fp64), so a window of
 // consecutive tiles is one contiguous block and a warp-wide load of 32
 // consecutive tiles coalesces into a few L2 requests.
-// DECAY kernels poll one predecessor record that its writer has just stored:
-// a 32-byte minimum stride keeps neighbouring tiles' records in different
-// sectors.  Generic kernels read windows of hundreds of records per poll:
-// packed records keep a window to a few lines.
-#ifndef PLR_STATUS_MIN_STRIDE_DEC
-#define PLR_STATUS_MIN_STRIDE_DEC 4
-#endif
-#ifndef PLR_STATUS_MIN_STRIDE_GEN
-#define PLR_STATUS_MIN_STRIDE_GEN 1
-#endif
+// Status records: NW 64-bit words at a power-of-two stride, placed at a
+// scattered slot (j * 0x9E3779B1) mod 2^c (odd multiplier: a bijection on the
+// 2^c slots), so the hundreds of records that concurrent look-backs poll are
+// spread over all L2 slices instead of hammering a few lines.
 template <typename A, int K, bool DEC>
 struct StatusLayout {
     static constexpr int NW = K * StatusIO<A>::kWords;
-    static constexpr int P2 = NW <= 1 ? 1 : NW <= 2 ? 2 : NW <= 4 ? 4 : 8;
-    static constexpr int MINS = DEC ? PLR_STATUS_MIN_STRIDE_DEC : PLR_STATUS_MIN_STRIDE_GEN;
-    static constexpr int STRIDE = P2 > MINS ? P2 : MINS;
+    static constexpr int STRIDE = NW <= 1 ? 1 : NW <= 2 ? 2 : NW <= 4 ? 4 : 8;
     static_assert(STRIDE * 8 <= kStatusMaxBytes, "status record stride");
 };
+__device__ __forceinline__ size_t status_slot(long long j, uint32_t mask) {
+#ifdef PLR_STATUS_LINEAR
+    (void)mask;
+    return (size_t)j;
+#else
+    return (size_t)(((uint32_t)j * 0x9E3779B1u) & mask);
+#endif
+}
 
 __device__ __forceinline__ void ld_relaxed_v2(const unsigned long long* p, unsigned long long& a,
                                               unsigned long long& b) {
@@ -196,11 +196,11 @@ __device__ __forceinline__ void ld_relaxed_v2(const unsigned long long* p, unsig
 // publish carry vector `val` of tile j with `tag`; lanes 0..NW-1 of the
 // calling warp each store one 64-bit word (single-copy atomic per word)
 template <typename A, int K, bool DEC>
-__device__ __forceinline__ void publish_status(unsigned long long* status, long long j, const A (&val)[K],
-                                               uint32_t tag, int lane) {
+__device__ __forceinline__ void publish_status(unsigned long long* status, uint32_t mask, long long j,
+                                               const A (&val)[K], uint32_t tag, int lane) {
     using SIO = StatusIO<A>;
     using SL = StatusLayout<A, K, DEC>;
-    unsigned long long* stj = status + (size_t)j * SL::STRIDE;
+    unsigned long long* stj = status + status_slot(j, mask) * SL::STRIDE;
     unsigned long long w[SL::NW];
 #pragma unroll
     for (int q = 0; q < K; q++) SIO::pack(val[q], tag, &w[q * SIO::kWords]);
@@ -212,12 +212,12 @@ __device__ __forceinline__ void publish_status(unsigned long long* status, long 
 // word carries its own tag, so 16-byte vector loads (two relaxed 64-bit
 // accesses) are as safe as scalar ones.
 template <typename A, int K, bool DEC>
-__device__ __forceinline__ int read_status(const unsigned long long* status, long long jj, A (&val)[K],
-                                           uint32_t tagA, uint32_t tagI) {
+__device__ __forceinline__ int read_status(const unsigned long long* status, uint32_t mask, long long jj,
+                                           A (&val)[K], uint32_t tagA, uint32_t tagI) {
     using SIO = StatusIO<A>;
     using SL = StatusLayout<A, K, DEC>;
     constexpr int NW = SL::NW;
-    const unsigned long long* sp = status + (size_t)jj * SL::STRIDE;
+    const unsigned long long* sp = status + status_slot(jj, mask) * SL::STRIDE;
     unsigned long long w[NW + 1];
 #pragma unroll
     for (int e = 0; e + 1 < NW + (NW & 1); e += 2) {
@@ -377,7 +377,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 A v[K];
                 if (lane == 0) {
                     int ns = 16;
-                    while (read_status<A, K, DEC>(prm.status, j - 1, v, tagA, tagI) != 2) {
+                    while (read_status<A, K, DEC>(prm.status, prm.status_mask, j - 1, v, tagA, tagI) != 2) {
                         __nanosleep(ns);
                         ns = ns < 256 ? 2 * ns : ns;
                     }
@@ -439,7 +439,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                         for (int q = 0; q < K; q++) v[t][q] = A(0);
                         if (t < tpl) {
                             const long long jj = j - 1 - (o + 32LL * t + lane);
-                            if (jj >= 0) st[t] = read_status<A, K, DEC>(prm.status, jj, v[t], tagA, tagI);
+                            if (jj >= 0) st[t] = read_status<A, K, DEC>(prm.status, prm.status_mask, jj, v[t], tagA, tagI);
                         }
                     }
                     int di = 1 << 30, dn = 1 << 30;              // lane's nearest inclusive / not-ready
@@ -536,7 +536,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 matvec_acc<A, K>(G, tb.Tm, Gp);                // G_j = A_j + T(m) G_{j-1}
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&carry_bar[slot]);
-                publish_status<A, K, DEC>(prm.status, j, G, tagI, lane);
+                publish_status<A, K, DEC>(prm.status, prm.status_mask, j, G, tagI, lane);
             } else {
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&carry_bar[slot]);
@@ -655,7 +655,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             A At[K];
 #pragma unroll
             for (int q = 0; q < K; q++) At[q] = shfl_idx(u_[q], W - 1);
-            publish_status<A, K, DEC>(prm.status, j, At, DEC ? 2u * prm.epoch + 1u : 2u * prm.epoch, lane);
+            publish_status<A, K, DEC>(prm.status, prm.status_mask, j, At, DEC ? 2u * prm.epoch + 1u : 2u * prm.epoch, lane);
         }
         // wagg is buffered per slot: its next writer (tile it+NS) runs after
         // every warp passed tile it+1's barrier

@@ -15,6 +15,7 @@ struct LaunchArgs {
     unsigned long long ticket_base;
     unsigned long long* ticket;
     unsigned long long* status;
+    uint32_t status_mask;
     uint32_t epoch;
     int decay;
     const void* x_hist;

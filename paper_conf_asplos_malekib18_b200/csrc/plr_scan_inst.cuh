@@ -26,8 +26,8 @@ namespace inst {
 #define PLR_GEN_D 3
 #define PLR_GEN_NL 2
 #define PLR_GEN_X 15
-#define PLR_GEN_W 8
-#define PLR_GEN_MINB 2
+#define PLR_GEN_W 16
+#define PLR_GEN_MINB 1
 #endif
 
 // S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
@@ -62,6 +62,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     prm.ticket_base = la.ticket_base;
     prm.ticket = la.ticket;
     prm.status = la.status;
+    prm.status_mask = la.status_mask;
     prm.epoch = la.epoch;
     prm.decay = la.decay;
     prm.x_hist = static_cast<const T*>(la.x_hist);
