@@ -118,9 +118,10 @@ plr_status plr_plan_factor_lists(const plr_plan* plan, int64_t m, void* out);
  * environment at plan creation (otherwise all zero): out[0] look-backs,
  * out[1] window polls, out[2] polls that folded nothing, out[3] summed
  * depth in tiles, out[4] SM cycles waiting for the tile's own aggregate,
- * out[5] cycles looking back, out[6] of which sleeping.  Synchronous;
+ * out[5] cycles looking back, out[6] of which sleeping, out[7] loading and
+ * classifying windows, out[8] folding.  Synchronous;
  * reset != 0 clears them.  Host memory. */
-plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out /* 8 */, int reset);
+plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out /* 16 */, int reset);
 
 /* y[0..n) = recurrence over x[0..n) with zero initial conditions.
  * x, y: device pointers of the plan's dtype. */

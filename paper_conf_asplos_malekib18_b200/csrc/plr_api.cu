@@ -364,8 +364,8 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     if ((e = cudaMalloc(&plan->d_hist, 64)) != cudaSuccess) return bail(e, "alloc hist");
     const char* st_env = std::getenv("PLR_STATS");
     if (st_env != nullptr && st_env[0] == '1') {
-        if ((e = cudaMalloc(&plan->d_stats, 64)) != cudaSuccess) return bail(e, "alloc stats");
-        if ((e = cudaMemset(plan->d_stats, 0, 64)) != cudaSuccess) return bail(e, "memset stats");
+        if ((e = cudaMalloc(&plan->d_stats, 128)) != cudaSuccess) return bail(e, "alloc stats");
+        if ((e = cudaMemset(plan->d_stats, 0, 128)) != cudaSuccess) return bail(e, "memset stats");
     }
     if ((e = cudaMemset(plan->d_hist, 0, 64)) != cudaSuccess) return bail(e, "memset hist");
     *out = plan;
@@ -395,11 +395,11 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
 plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out, int reset) {
     if (plan == nullptr || out == nullptr) return fail(PLR_ERR_INVALID_ARG, "null argument");
     if (plan->d_stats == nullptr) {
-        memset(out, 0, 8 * sizeof(uint64_t));
+        memset(out, 0, 16 * sizeof(uint64_t));
         return PLR_OK;
     }
     CUDA_TRY(cudaMemcpy(out, plan->d_stats, 64, cudaMemcpyDeviceToHost), "stats copy");
-    if (reset) CUDA_TRY(cudaMemset(plan->d_stats, 0, 64), "stats reset");
+    if (reset) CUDA_TRY(cudaMemset(plan->d_stats, 0, 128), "stats reset");
     return PLR_OK;
 }
 

@@ -425,8 +425,10 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #endif
                 int ns = PLR_LB_NS0;
                 unsigned long long n_win = 0, n_wait = 0;
+                long long c_load = 0, c_fold = 0;
                 for (;;) {
                     n_win++;
+                    const long long cl0 = clock64();
                     const int tpl = 1 << ltpl;
                     // lane-interleaved window: distance d = o + 32 t + lane, t < tpl,
                     // so every warp-wide load reads 32 consecutive tiles
@@ -452,6 +454,8 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     const int dN = __reduce_min_sync(0xffffffffu, (unsigned)dn);
                     const bool found = dI < dN;
                     const int e = found ? dI + 1 : (dN < (1 << 30) ? dN : 32 * tpl);   // tiles to fold now
+                    const long long cl1 = clock64();
+                    c_load += cl1 - cl0;
                     if (e > 0) {
                         // per-lane Horner over t (stride 32 tiles), then a tree over lanes
                         A r[K];
@@ -480,6 +484,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
                         for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
                         matvec_acc<A, K>(acc, Tacc, R);
+                        c_fold += clock64() - cl1;
                         if (found) break;
                         // skip the folded tiles: Tacc *= T(e m) (binary powers)
 #pragma unroll 1
@@ -519,6 +524,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     atomicAdd(&prm.stats[4], (unsigned long long)(c_agg - c_start));    // cycles waiting own A
                     atomicAdd(&prm.stats[5], (unsigned long long)(clock64() - c_agg));  // cycles looking back
                     atomicAdd(&prm.stats[6], (unsigned long long)c_wait);               // of which sleeping
+                    atomicAdd(&prm.stats[7], (unsigned long long)c_load);               // loading + classifying windows
+                    atomicAdd(&prm.stats[8], (unsigned long long)c_fold);               // folding
+
                 }
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = acc[q];

@@ -22,10 +22,10 @@ namespace inst {
 #define PLR_DEC_MINB 3
 #endif
 #ifndef PLR_GEN_S
-#define PLR_GEN_S 6
-#define PLR_GEN_D 3
+#define PLR_GEN_S 3
+#define PLR_GEN_D 1
 #define PLR_GEN_NL 2
-#define PLR_GEN_X 15
+#define PLR_GEN_X 31
 #define PLR_GEN_W 16
 #define PLR_GEN_MINB 1
 #endif

@@ -32,8 +32,9 @@ for name in names:
     st = plan.debug_stats()
     lb = max(1, st["lookbacks"])
     print("%-7s %8.3f ms %7.1f GB/s  lb/launch %d  polls/lb %.2f  waits/lb %.2f  depth/lb %.1f  "
-          "cyc: agg %.0f lb %.0f sleep %.0f  info %s" % (
+          "cyc: agg %.0f lb %.0f sleep %.0f load %.0f fold %.0f  info %s" % (
               name, ms, n * 8 / ms / 1e6, st["lookbacks"] // reps, st["windows"] / lb, st["waits"] / lb,
               st["depth_sum"] / lb, st["cyc_agg"] / lb, st["cyc_lookback"] / lb, st["cyc_sleep"] / lb,
+              st["cyc_load"] / lb, st["cyc_fold"] / lb,
               {k: plan.info[k] for k in ("ctas_per_sm", "cls")}), flush=True)
     plan.close()
