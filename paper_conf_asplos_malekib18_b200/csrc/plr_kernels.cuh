@@ -235,6 +235,36 @@ __device__ __forceinline__ int read_status(const unsigned long long* status, uin
     return allI ? 2 : (allA ? 1 : 0);
 }
 
+// Split form of read_status for windows: issue every load of the window
+// first, classify afterwards, so the loads of all tiles are in flight
+// together (one L2 round trip per window, not one per tile).
+template <typename A, int K, bool DEC>
+__device__ __forceinline__ void load_status_raw(const unsigned long long* status, uint32_t mask, long long jj,
+                                                unsigned long long (&w)[StatusLayout<A, K, DEC>::NW]) {
+    using SL = StatusLayout<A, K, DEC>;
+    constexpr int NW = SL::NW;
+    const unsigned long long* sp = status + status_slot(jj, mask) * SL::STRIDE;
+#pragma unroll
+    for (int e = 0; e < NW; e += 2) {
+        if (e + 1 < NW) ld_relaxed_v2(sp + e, w[e], w[e + 1]);
+        else w[e] = ld_relaxed(sp + e);
+    }
+}
+template <typename A, int K, bool DEC>
+__device__ __forceinline__ int classify_status(const unsigned long long (&w)[StatusLayout<A, K, DEC>::NW],
+                                               A (&val)[K], uint32_t tagA, uint32_t tagI) {
+    using SIO = StatusIO<A>;
+    bool allI = true, allA = true;
+#pragma unroll
+    for (int q = 0; q < K; q++) {
+        const bool i1 = SIO::unpack(&w[q * SIO::kWords], tagI, val[q]);
+        const bool a1 = SIO::unpack(&w[q * SIO::kWords], tagA, val[q]);
+        allI = allI && i1;
+        allA = allA && a1;
+    }
+    return allI ? 2 : (allA ? 1 : 0);
+}
+
 // ------------------------------------------------------ shared memory ------
 template <typename T, typename A, int K, int X, int W, int S, int D>
 struct Layout {
@@ -432,6 +462,13 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     const int tpl = 1 << ltpl;
                     // lane-interleaved window: distance d = o + 32 t + lane, t < tpl,
                     // so every warp-wide load reads 32 consecutive tiles
+                    using SLw = StatusLayout<A, K, DEC>;
+                    unsigned long long raw[kTPL][SLw::NW];
+#pragma unroll
+                    for (int t = 0; t < kTPL; t++) {             // all loads in flight together
+                        const long long jj = j - 1 - (o + 32LL * t + lane);
+                        if (t < tpl && jj >= 0) load_status_raw<A, K, DEC>(prm.status, prm.status_mask, jj, raw[t]);
+                    }
                     A v[kTPL][K];
                     int st[kTPL];
 #pragma unroll
@@ -439,10 +476,8 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                         st[t] = 2;
 #pragma unroll
                         for (int q = 0; q < K; q++) v[t][q] = A(0);
-                        if (t < tpl) {
-                            const long long jj = j - 1 - (o + 32LL * t + lane);
-                            if (jj >= 0) st[t] = read_status<A, K, DEC>(prm.status, prm.status_mask, jj, v[t], tagA, tagI);
-                        }
+                        const long long jj = j - 1 - (o + 32LL * t + lane);
+                        if (t < tpl && jj >= 0) st[t] = classify_status<A, K, DEC>(raw[t], v[t], tagA, tagI);
                     }
                     int di = 1 << 30, dn = 1 << 30;              // lane's nearest inclusive / not-ready
 #pragma unroll
