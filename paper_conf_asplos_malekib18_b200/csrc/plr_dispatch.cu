@@ -6,12 +6,14 @@ namespace plr {
 Geometry class_geometry(bool decay) {
     // x elements per thread (odd: conflict-free strided smem access) and W
     // compute warps per config; the ring depth is reported by scan_stages()
-    return decay ? Geometry{inst::CfgDec::X, inst::CfgDec::W, inst::CfgDec::S}
-                 : Geometry{inst::CfgGen::X, inst::CfgGen::W, inst::CfgGen::S};
+    if (decay) return Geometry{inst::CfgDec::X, inst::CfgDec::W, inst::CfgDec::S};
+    if (PLR_GEN_TMEM) return Geometry{PLR_TM_X, PLR_TM_W, PLR_TM_SL};
+    return Geometry{inst::CfgGen::X, inst::CfgGen::W, inst::CfgGen::S};
 }
 
 int scan_stages(const PlanTables& pt) {
-    return pt.decay_flag ? inst::CfgDec::S : inst::CfgGen::S;
+    if (pt.decay_flag) return inst::CfgDec::S;
+    return PLR_GEN_TMEM ? PLR_TM_SL : inst::CfgGen::S;
 }
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la) {

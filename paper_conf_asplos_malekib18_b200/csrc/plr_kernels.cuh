@@ -265,6 +265,152 @@ __device__ __forceinline__ int classify_status(const unsigned long long (&w)[Sta
     return allI ? 2 : (allA ? 1 : 0);
 }
 
+
+// Generic look-back: fold the tiles j-1, j-2, ...
+// nearest first, G_{j-1} = sum_d T(d m) v_{j-1-d}, v = aggregate for "P"
+// tiles and the inclusive carry of the first "I" tile.  Each poll reads a
+// lane-interleaved window (all loads in flight together), folds its ready
+// prefix (up to the first not-ready or first inclusive tile) and never
+// re-reads folded tiles.  Called by one full warp.
+template <typename T, typename A, int K, bool DEC>
+__device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, const Tables<T, A>& tb, long long j,
+                                                 int lane, uint32_t tagA, uint32_t tagI, A (&Gp)[K],
+                                                 long long c_start = 0, long long c_agg = 0) {
+    long long c_wait = 0;
+    // tiles per lane of a full window: 8 for small records, 4 when a record
+    // has more than 2 words (keeps the window's registers in check)
+    constexpr int kT = StatusLayout<A, K, DEC>::NW <= 2 ? kTPL : kTPL / 2;
+    constexpr int kLogT = kT == 8 ? 3 : 2;
+    A acc[K];
+    A Tacc[K * kMaxK];
+#pragma unroll
+    for (int q = 0; q < K; q++) {
+        acc[q] = A(0);
+#pragma unroll
+        for (int r = 0; r < kMaxK; r++) Tacc[q * kMaxK + r] = (q == r) ? A(1) : A(0);
+    }
+    long long o = 0;                   // distance of the first unfolded tile from j-1
+#ifndef PLR_LB_LTPL0
+#define PLR_LB_LTPL0 3
+#endif
+    int ltpl = PLR_LB_LTPL0 < kLogT ? PLR_LB_LTPL0 : kLogT;   // log2 tiles per lane of the first window
+#ifndef PLR_LB_NS0
+#define PLR_LB_NS0 32
+#endif
+    int ns = PLR_LB_NS0;
+    unsigned long long n_win = 0, n_wait = 0;
+    long long c_load = 0, c_fold = 0;
+    for (;;) {
+        n_win++;
+        const long long cl0 = clock64();
+        const int tpl = 1 << ltpl;
+        // lane-interleaved window: distance d = o + 32 t + lane, t < tpl,
+        // so every warp-wide load reads 32 consecutive tiles
+        using SLw = StatusLayout<A, K, DEC>;
+        unsigned long long raw[kT][SLw::NW];
+#pragma unroll
+        for (int t = 0; t < kT; t++) {             // all loads in flight together
+            const long long jj = j - 1 - (o + 32LL * t + lane);
+            if (t < tpl && jj >= 0) load_status_raw<A, K, DEC>(prm.status, prm.status_mask, jj, raw[t]);
+        }
+        A v[kT][K];
+        int st[kT];
+#pragma unroll
+        for (int t = 0; t < kT; t++) {
+            st[t] = 2;
+#pragma unroll
+            for (int q = 0; q < K; q++) v[t][q] = A(0);
+            const long long jj = j - 1 - (o + 32LL * t + lane);
+            if (t < tpl && jj >= 0) st[t] = classify_status<A, K, DEC>(raw[t], v[t], tagA, tagI);
+        }
+        int di = 1 << 30, dn = 1 << 30;              // lane's nearest inclusive / not-ready
+#pragma unroll
+        for (int t = kT - 1; t >= 0; t--) {
+            if (t < tpl && st[t] == 2) di = 32 * t + lane;
+            if (t < tpl && st[t] == 0) dn = 32 * t + lane;
+        }
+        const int dI = __reduce_min_sync(0xffffffffu, (unsigned)di);
+        const int dN = __reduce_min_sync(0xffffffffu, (unsigned)dn);
+        const bool found = dI < dN;
+        const int e = found ? dI + 1 : (dN < (1 << 30) ? dN : 32 * tpl);   // tiles to fold now
+        const long long cl1 = clock64();
+        c_load += cl1 - cl0;
+        if (e > 0) {
+            // per-lane Horner over t (stride 32 tiles), then a tree over lanes
+            A r[K];
+#pragma unroll
+            for (int q = 0; q < K; q++) r[q] = A(0);
+#pragma unroll
+            for (int t = kT - 1; t >= 0; t--) {
+                if (t < tpl && 32 * t + lane < e) {
+                    A nr[K];
+#pragma unroll
+                    for (int q = 0; q < K; q++) nr[q] = v[t][q];
+                    matvec_acc<A, K>(nr, tb.Tpow[5], r);           // T(32 m)
+#pragma unroll
+                    for (int q = 0; q < K; q++) r[q] = nr[q];
+                }
+            }
+            // R = sum_l T(l m) r_l, T(m 2^s) = Tpow[s]
+#pragma unroll
+            for (int s2 = 0; s2 < 5; s2++) {
+                A o2[K];
+#pragma unroll
+                for (int q = 0; q < K; q++) o2[q] = shfl_down(r[q], 1 << s2);
+                matvec_acc<A, K>(r, tb.Tpow[s2], o2);
+            }
+            A R[K];
+#pragma unroll
+            for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
+            matvec_acc<A, K>(acc, Tacc, R);
+            c_fold += clock64() - cl1;
+            if (found) break;
+            // skip the folded tiles: Tacc *= T(e m) (binary powers)
+#pragma unroll 1
+            for (int s2 = 0; s2 < 9; s2++) {
+                if (!((e >> s2) & 1)) continue;
+                A nt[K * kMaxK];
+#pragma unroll
+                for (int q = 0; q < K; q++)
+#pragma unroll
+                    for (int c2 = 0; c2 < K; c2++) {
+                        A a2 = A(0);
+#pragma unroll
+                        for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], tb.Tpow[s2][t * kMaxK + c2], a2);
+                        nt[q * kMaxK + c2] = a2;
+                    }
+#pragma unroll
+                for (int q = 0; q < K; q++)
+#pragma unroll
+                    for (int c2 = 0; c2 < K; c2++) Tacc[q * kMaxK + c2] = nt[q * kMaxK + c2];
+            }
+            o += e;
+            ns = PLR_LB_NS0;
+            if (dN >= (1 << 30)) ltpl = kLogT;         // nothing pending: widen to the full window
+        } else {
+            n_wait++;                                  // nearest tile not ready yet
+            const long long cw = clock64();
+            __nanosleep(ns);
+            c_wait += clock64() - cw;
+            ns = ns < 512 ? 2 * ns : ns;
+        }
+    }
+    if (prm.stats != nullptr && lane == 0) {
+        atomicAdd(&prm.stats[0], 1ull);                // look-backs
+        atomicAdd(&prm.stats[1], n_win);               // window polls
+        atomicAdd(&prm.stats[2], n_wait);              // polls that folded nothing
+        atomicAdd(&prm.stats[3], (unsigned long long)(o + 1));  // depth folded (approx.)
+        atomicAdd(&prm.stats[4], (unsigned long long)(c_agg - c_start));    // cycles waiting own A
+        atomicAdd(&prm.stats[5], (unsigned long long)(clock64() - c_agg));  // cycles looking back
+        atomicAdd(&prm.stats[6], (unsigned long long)c_wait);               // of which sleeping
+        atomicAdd(&prm.stats[7], (unsigned long long)c_load);               // loading + classifying windows
+        atomicAdd(&prm.stats[8], (unsigned long long)c_fold);               // folding
+
+    }
+#pragma unroll
+    for (int q = 0; q < K; q++) Gp[q] = acc[q];
+}
+
 // ------------------------------------------------------ shared memory ------
 template <typename T, typename A, int K, int X, int W, int S, int D>
 struct Layout {
@@ -436,135 +582,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     mbar_wait(&agg_bar[nx % NS], (uint32_t)((nx / NS) & 1));
                 }
                 const long long c_agg = clock64();
-                long long c_wait = 0;
-                A acc[K];
-                A Tacc[K * kMaxK];
-#pragma unroll
-                for (int q = 0; q < K; q++) {
-                    acc[q] = A(0);
-#pragma unroll
-                    for (int r = 0; r < kMaxK; r++) Tacc[q * kMaxK + r] = (q == r) ? A(1) : A(0);
-                }
-                long long o = 0;                   // distance of the first unfolded tile from j-1
-#ifndef PLR_LB_LTPL0
-#define PLR_LB_LTPL0 3
-#endif
-                int ltpl = PLR_LB_LTPL0;           // log2 tiles per lane: 2 (64-tile window), then 8
-#ifndef PLR_LB_NS0
-#define PLR_LB_NS0 32
-#endif
-                int ns = PLR_LB_NS0;
-                unsigned long long n_win = 0, n_wait = 0;
-                long long c_load = 0, c_fold = 0;
-                for (;;) {
-                    n_win++;
-                    const long long cl0 = clock64();
-                    const int tpl = 1 << ltpl;
-                    // lane-interleaved window: distance d = o + 32 t + lane, t < tpl,
-                    // so every warp-wide load reads 32 consecutive tiles
-                    using SLw = StatusLayout<A, K, DEC>;
-                    unsigned long long raw[kTPL][SLw::NW];
-#pragma unroll
-                    for (int t = 0; t < kTPL; t++) {             // all loads in flight together
-                        const long long jj = j - 1 - (o + 32LL * t + lane);
-                        if (t < tpl && jj >= 0) load_status_raw<A, K, DEC>(prm.status, prm.status_mask, jj, raw[t]);
-                    }
-                    A v[kTPL][K];
-                    int st[kTPL];
-#pragma unroll
-                    for (int t = 0; t < kTPL; t++) {
-                        st[t] = 2;
-#pragma unroll
-                        for (int q = 0; q < K; q++) v[t][q] = A(0);
-                        const long long jj = j - 1 - (o + 32LL * t + lane);
-                        if (t < tpl && jj >= 0) st[t] = classify_status<A, K, DEC>(raw[t], v[t], tagA, tagI);
-                    }
-                    int di = 1 << 30, dn = 1 << 30;              // lane's nearest inclusive / not-ready
-#pragma unroll
-                    for (int t = kTPL - 1; t >= 0; t--) {
-                        if (t < tpl && st[t] == 2) di = 32 * t + lane;
-                        if (t < tpl && st[t] == 0) dn = 32 * t + lane;
-                    }
-                    const int dI = __reduce_min_sync(0xffffffffu, (unsigned)di);
-                    const int dN = __reduce_min_sync(0xffffffffu, (unsigned)dn);
-                    const bool found = dI < dN;
-                    const int e = found ? dI + 1 : (dN < (1 << 30) ? dN : 32 * tpl);   // tiles to fold now
-                    const long long cl1 = clock64();
-                    c_load += cl1 - cl0;
-                    if (e > 0) {
-                        // per-lane Horner over t (stride 32 tiles), then a tree over lanes
-                        A r[K];
-#pragma unroll
-                        for (int q = 0; q < K; q++) r[q] = A(0);
-#pragma unroll
-                        for (int t = kTPL - 1; t >= 0; t--) {
-                            if (t < tpl && 32 * t + lane < e) {
-                                A nr[K];
-#pragma unroll
-                                for (int q = 0; q < K; q++) nr[q] = v[t][q];
-                                matvec_acc<A, K>(nr, tb.Tpow[5], r);           // T(32 m)
-#pragma unroll
-                                for (int q = 0; q < K; q++) r[q] = nr[q];
-                            }
-                        }
-                        // R = sum_l T(l m) r_l, T(m 2^s) = Tpow[s]
-#pragma unroll
-                        for (int s2 = 0; s2 < 5; s2++) {
-                            A o2[K];
-#pragma unroll
-                            for (int q = 0; q < K; q++) o2[q] = shfl_down(r[q], 1 << s2);
-                            matvec_acc<A, K>(r, tb.Tpow[s2], o2);
-                        }
-                        A R[K];
-#pragma unroll
-                        for (int q = 0; q < K; q++) R[q] = shfl_idx(r[q], 0);
-                        matvec_acc<A, K>(acc, Tacc, R);
-                        c_fold += clock64() - cl1;
-                        if (found) break;
-                        // skip the folded tiles: Tacc *= T(e m) (binary powers)
-#pragma unroll 1
-                        for (int s2 = 0; s2 < 9; s2++) {
-                            if (!((e >> s2) & 1)) continue;
-                            A nt[K * kMaxK];
-#pragma unroll
-                            for (int q = 0; q < K; q++)
-#pragma unroll
-                                for (int c2 = 0; c2 < K; c2++) {
-                                    A a2 = A(0);
-#pragma unroll
-                                    for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], tb.Tpow[s2][t * kMaxK + c2], a2);
-                                    nt[q * kMaxK + c2] = a2;
-                                }
-#pragma unroll
-                            for (int q = 0; q < K; q++)
-#pragma unroll
-                                for (int c2 = 0; c2 < K; c2++) Tacc[q * kMaxK + c2] = nt[q * kMaxK + c2];
-                        }
-                        o += e;
-                        ns = PLR_LB_NS0;
-                        if (dN >= (1 << 30)) ltpl = 3;             // nothing pending: widen to 256 tiles
-                    } else {
-                        n_wait++;                                  // nearest tile not ready yet
-                        const long long cw = clock64();
-                        __nanosleep(ns);
-                        c_wait += clock64() - cw;
-                        ns = ns < 512 ? 2 * ns : ns;
-                    }
-                }
-                if (prm.stats != nullptr && lane == 0) {
-                    atomicAdd(&prm.stats[0], 1ull);                // look-backs
-                    atomicAdd(&prm.stats[1], n_win);               // window polls
-                    atomicAdd(&prm.stats[2], n_wait);              // polls that folded nothing
-                    atomicAdd(&prm.stats[3], (unsigned long long)(o + 1));  // depth folded (approx.)
-                    atomicAdd(&prm.stats[4], (unsigned long long)(c_agg - c_start));    // cycles waiting own A
-                    atomicAdd(&prm.stats[5], (unsigned long long)(clock64() - c_agg));  // cycles looking back
-                    atomicAdd(&prm.stats[6], (unsigned long long)c_wait);               // of which sleeping
-                    atomicAdd(&prm.stats[7], (unsigned long long)c_load);               // loading + classifying windows
-                    atomicAdd(&prm.stats[8], (unsigned long long)c_fold);               // folding
-
-                }
-#pragma unroll
-                for (int q = 0; q < K; q++) Gp[q] = acc[q];
+                lookback_generic<T, A, K, DEC>(prm, tb, j, lane, tagA, tagI, Gp, c_start, c_agg);
             }
             // the tile's own aggregate (phase A) is needed for its inclusive carry
             if (j == 0 || DEC) mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));

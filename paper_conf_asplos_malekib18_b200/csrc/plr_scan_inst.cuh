@@ -3,6 +3,7 @@
 // per-type .cu files so the instantiations compile in parallel.
 #pragma once
 #include "plr_kernels.cuh"
+#include "plr_kernels_tmem.cuh"
 #include "plr_launch.h"
 
 namespace plr {
@@ -29,6 +30,19 @@ namespace inst {
 #define PLR_GEN_W 16
 #define PLR_GEN_MINB 1
 #endif
+// generic classes use the TMEM-parking kernel (plr_kernels_tmem.cuh) unless
+// PLR_GEN_TMEM=0: X, W, NL as below, SL load + ST store stages, as many
+// parked tiles as fit in 512 TMEM columns (max 8)
+#ifndef PLR_GEN_TMEM
+#define PLR_GEN_TMEM 1
+#endif
+#ifndef PLR_TM_X
+#define PLR_TM_X 15
+#define PLR_TM_W 16
+#define PLR_TM_NL 2
+#define PLR_TM_SL 3
+#define PLR_TM_ST 2
+#endif
 
 // S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
 // W compute warps (tile m = 32 W X)
@@ -41,19 +55,41 @@ struct Cfg {
 using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true>;
 using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false>;
 
+template <typename T, typename A, int K>
+struct TmCfg {
+    static constexpr int X = PLR_TM_X, W = PLR_TM_W, NL = PLR_TM_NL, SL = PLR_TM_SL, ST = PLR_TM_ST;
+    static constexpr int CW = dev::TmemCols<A, K, X>::CW;
+    static constexpr int NT0 = 512 / ((W / 4) * CW);
+    static constexpr int NT = NT0 > 8 ? 8 : NT0;
+};
+
 template <typename T, typename A, class C, int K, int P, bool STORE>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
-    auto kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB>;
-    const size_t smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
-    constexpr int threads = (C::W + 1 + C::NL) * 32;
+    constexpr bool tmem = PLR_GEN_TMEM && !C::DEC;
+    size_t smem;
+    int threads;
+    void (*kern)(const ScanParams<T, A>);
+    if constexpr (tmem) {
+        using TC = TmCfg<T, A, K>;
+        kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, STORE>;
+        smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
+        threads = (TC::W + 1 + TC::NL) * 32;
+    } else {
+        kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB>;
+        smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
+        threads = (C::W + 1 + C::NL) * 32;
+    }
     static bool configured = false;
     if (!configured) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         configured = true;
     }
-    if (la.occupancy_out != nullptr)    // occupancy query: report CTAs/SM, do not launch
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, threads, smem);
+    if (la.occupancy_out != nullptr) {  // occupancy query: report CTAs/SM, do not launch
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, threads, smem);
+        if (tmem && *la.occupancy_out > 1) *la.occupancy_out = 1;   // 512 TMEM columns per CTA
+        return e;
+    }
     ScanParams<T, A> prm;
     prm.x = static_cast<const T*>(la.x);
     prm.y = static_cast<T*>(la.y);
