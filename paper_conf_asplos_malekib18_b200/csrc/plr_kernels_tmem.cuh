@@ -227,6 +227,10 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 }
             }
         } else if (lane == 1) {                                     // storer
+            // up to ST-1 bulk stores in flight; a stage is handed back to the
+            // compute warps once the bulk store has finished reading it
+            int pend[ST];
+            int np = 0;
             for (int t = 0;; t++) {
                 const int sT = t % ST;
                 mbar_wait(&full_T[sT], (uint32_t)((t / ST) & 1));
@@ -235,11 +239,20 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 if (STORE && !(jt == ntiles - 1 && last_ragged)) {
                     bulk_store(prm.y + (size_t)jt * M, tstage + (size_t)sT * M, M * sizeof(T), pol);
                     bulk_commit();
-                    bulk_wait_read<0>();                            // stage read: compute may refill it
+                    pend[np++] = sT;
+                    if (np > ST - 1) {
+                        bulk_wait_read<ST - 1>();                   // the oldest store has read its stage
+                        mbar_arrive(&empty_T[pend[0]]);
+#pragma unroll
+                        for (int q = 0; q + 1 < ST; q++) pend[q] = pend[q + 1];
+                        np--;
+                    }
+                } else {
+                    mbar_arrive(&empty_T[sT]);                      // nothing read from this stage
                 }
-                mbar_arrive(&empty_T[sT]);
             }
             bulk_wait_all<0>();
+            for (int q = 0; q < np; q++) mbar_arrive(&empty_T[pend[q]]);
         }
         return;
     }
@@ -460,8 +473,9 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     for (; nb < na; nb++) phaseB(nb, slot_tile[nb % NT]);      // drain
     // stop markers: the storer, and look-back warps waiting beyond the stop
     {
+        // no wait for the stage: only its id slot is written, and the storer
+        // (which is at tile >= nb-2) has long read the previous id of it
         const int sT = nb % ST;
-        mbar_wait(&empty_T[sT], (uint32_t)(((nb / ST) & 1) ^ 1));
         if (tid == 0) store_tile[sT] = ntiles;
         mbar_arrive(&full_T[sT]);
     }

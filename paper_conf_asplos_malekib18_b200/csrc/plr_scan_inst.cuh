@@ -41,7 +41,7 @@ namespace inst {
 #define PLR_TM_W 16
 #define PLR_TM_NL 2
 #define PLR_TM_SL 3
-#define PLR_TM_ST 2
+#define PLR_TM_ST 3
 #endif
 
 // S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
