@@ -18,7 +18,7 @@ constexpr int kHalo = 4;            // words in front of each stage: x_{-4}..x_{
 constexpr int kMaxX = 31;
 constexpr int kMaxW = 16;
 constexpr int kStatusWords = 4;     // u64 status words per tile (>= kMaxK)
-constexpr int kStatusMaxBytes = 64;  // bytes per status slot the plan allocates (max record stride)
+constexpr int kStatusMaxBytes = 128; // bytes per status slot the plan allocates (max record stride)
 constexpr int kAug = 8;             // augmented state slots: x_{-4..-1}, y_{-4..-1}
 constexpr int kTPL = 8;             // look-back: tiles per lane in a wide window (2^3)
 

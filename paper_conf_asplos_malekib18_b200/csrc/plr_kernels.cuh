@@ -173,10 +173,14 @@ template <> struct StatusIO<double> {
 // scattered slot (j * 0x9E3779B1) mod 2^c (odd multiplier: a bijection on the
 // 2^c slots), so the hundreds of records that concurrent look-backs poll are
 // spread over all L2 slices instead of hammering a few lines.
+#ifndef PLR_STATUS_MIN_STRIDE
+#define PLR_STATUS_MIN_STRIDE 4      // words: one 32-byte sector per record at least
+#endif
 template <typename A, int K, bool DEC>
 struct StatusLayout {
     static constexpr int NW = K * StatusIO<A>::kWords;
-    static constexpr int STRIDE = NW <= 1 ? 1 : NW <= 2 ? 2 : NW <= 4 ? 4 : 8;
+    static constexpr int P2 = NW <= 1 ? 1 : NW <= 2 ? 2 : NW <= 4 ? 4 : 8;
+    static constexpr int STRIDE = P2 > PLR_STATUS_MIN_STRIDE ? P2 : PLR_STATUS_MIN_STRIDE;
     static_assert(STRIDE * 8 <= kStatusMaxBytes, "status record stride");
 };
 __device__ __forceinline__ size_t status_slot(long long j, uint32_t mask) {
