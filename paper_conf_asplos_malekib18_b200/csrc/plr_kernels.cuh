@@ -295,7 +295,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
     }
     long long o = 0;                   // distance of the first unfolded tile from j-1
 #ifndef PLR_LB_LTPL0
-#define PLR_LB_LTPL0 3
+#define PLR_LB_LTPL0 1
 #endif
     int ltpl = PLR_LB_LTPL0 < kLogT ? PLR_LB_LTPL0 : kLogT;   // log2 tiles per lane of the first window
 #ifndef PLR_LB_NS0

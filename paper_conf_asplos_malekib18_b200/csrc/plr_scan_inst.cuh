@@ -59,8 +59,11 @@ template <typename T, typename A, int K>
 struct TmCfg {
     static constexpr int X = PLR_TM_X, W = PLR_TM_W, NL = PLR_TM_NL, SL = PLR_TM_SL, ST = PLR_TM_ST;
     static constexpr int CW = dev::TmemCols<A, K, X>::CW;
+#ifndef PLR_TM_NTMAX
+#define PLR_TM_NTMAX 8
+#endif
     static constexpr int NT0 = 512 / ((W / 4) * CW);
-    static constexpr int NT = NT0 > 8 ? 8 : NT0;
+    static constexpr int NT = NT0 > PLR_TM_NTMAX ? PLR_TM_NTMAX : NT0;
 };
 
 template <typename T, typename A, class C, int K, int P, bool STORE>

@@ -1,6 +1,6 @@
 set -x
 rm -f gpurun_out/lbstats.log
-for v in "" _u8 _u16; do
+for v in "" _nt7 _nt5; do
   echo "== variant '$v'" >> gpurun_out/lbstats.log
-  PLR_LIB=$PWD/paper_conf_asplos_malekib18_b200/libplr_b200$v.so timeout 300 python tools/lookback_stats.py $((1<<30)) prefix,tuple2,tuple3,lp1,lp3,hp3 >> gpurun_out/lbstats.log 2>&1
+  PLR_LIB=$PWD/paper_conf_asplos_malekib18_b200/libplr_b200$v.so timeout 300 python tools/lookback_stats.py $((1<<30)) prefix,tuple2,tuple3 >> gpurun_out/lbstats.log 2>&1
 done
