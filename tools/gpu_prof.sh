@@ -1,2 +1,2 @@
 set -x
-bash tools/ncu_profile.sh r01b "prefix tuple2 lp1 hp3"
+bash tools/ncu_profile.sh r01b "prefix tuple2"
