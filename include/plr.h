@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define PLR_ABI_VERSION 1
+#define PLR_ABI_VERSION 2
 #define PLR_MAX_K 4            /* maximum order k supported by the kernels      */
 #define PLR_MAX_P 3            /* maximum feed-forward order p                  */
 #define PLR_PAYLOAD_BYTES 64   /* one rank's end-state record, see plr_reduce   */
@@ -90,6 +90,10 @@ typedef struct {
     size_t scratch_bytes;      /* device bytes the plan owns                      */
     int ctas_per_sm;
     int num_sms;
+    int const_sig;             /* != 0: the scan kernel has this signature's tables as
+                                  compile-time constants (the generator's per-signature
+                                  code); 0: tables read from the
+                                  kernel parameters                                   */
 } plr_plan_info;
 
 /* Create a plan.  a[0..p] = (a0, a-1, ..., a-p) (p = feed-forward order, so

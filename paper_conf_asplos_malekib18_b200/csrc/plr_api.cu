@@ -47,6 +47,7 @@ struct plr_plan {
     void* d_lane = nullptr;
     float* d_fix = nullptr;
     bool dirty = false;
+    bool sig_kernel = false;            // launch the compile-time signature kernel (pt.sig_id)
     unsigned long long* d_stats = nullptr;   // look-back counters when PLR_STATS=1
     // sharded path scratch
     unsigned char* d_send = nullptr;
@@ -234,6 +235,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.lane_T = plan->d_lane;
     la.stats = plan->d_stats;
     la.grid = (int)grid;
+    la.sig = plan->sig_kernel ? plan->pt.sig_id : 0;
     la.store = store;
     la.stream = stream;
     cudaError_t e = launch_scan(plan->pt, la);
@@ -331,6 +333,11 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
         delete plan;
         return fail(st, why);
     }
+    // compile-time signature kernels (plr_constsig.cuh) unless the ablation
+    // switches are set: PLR_FORCE_GENERIC=1 (all specialisations off) or
+    // PLR_NO_CONSTSIG=1 (tables from kernel parameters only)
+    const char* ncs = std::getenv("PLR_NO_CONSTSIG");
+    plan->sig_kernel = !force_generic && !(ncs != nullptr && ncs[0] == '1') && plan->pt.sig_id != 0;
     plan->n_max = n_max;
     if (n_max == 0) {                      // host-only plan: planner tables, no device state
         *out = plan;
@@ -397,6 +404,7 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
                           (size_t)plan->pt.fixup_len * kAug * 4 + 64;
     info->ctas_per_sm = plan->ctas_per_sm;
     info->num_sms = plan->num_sms;
+    info->const_sig = plan->sig_kernel ? plan->pt.sig_id : 0;
     return PLR_OK;
 }
 

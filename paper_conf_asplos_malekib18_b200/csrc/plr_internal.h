@@ -76,6 +76,7 @@ struct PlanTables {
     int decay_flag;
     int acc64;                           // float: accumulate recurrence + carries in fp64
     double cond_bound;                   // eps32 * sum|a| * (sum|g|)^2 (float)
+    int sig_id;                          // compile-time signature kernel (plr_constsig.cuh), 0 = none
     Tables<uint32_t, uint32_t> ti;       // int32 ring
     Tables<float, float> tf;             // fp32, fp32 accumulation
     Tables<float, double> td;            // fp32, fp64 accumulation

@@ -369,8 +369,9 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
             matvec_acc<A, K>(acc, Tacc, R);
             c_fold += clock64() - cl1;
             if (found) break;
-            // skip the folded tiles: Tacc *= T(e m) (binary powers)
-#pragma unroll 1
+            // skip the folded tiles: Tacc *= T(e m) (binary powers; unrolled so
+            // compile-time tables fold)
+#pragma unroll
             for (int s2 = 0; s2 < 9; s2++) {
                 if (!((e >> s2) & 1)) continue;
                 A nt[K * kMaxK];

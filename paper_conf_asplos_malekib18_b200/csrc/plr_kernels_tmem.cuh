@@ -18,6 +18,7 @@
 //   warp W lane 1  storer: cp.async.bulk stores of finished tiles
 //   warps W+1..    look-back (a5), taking turns over the CTA's tiles
 #pragma once
+#include "plr_constsig.cuh"
 #include "plr_kernels.cuh"
 
 namespace plr {
@@ -148,7 +149,7 @@ struct LayoutT {
 template <typename A, int K, int X>
 struct TmemCols { static constexpr int CW = X + K * AWords<A>::N; };
 
-template <typename T, typename A, int K, int P, int X, int W, int SL, int ST, int NT, int NL, bool STORE>
+template <typename T, typename A, int K, int P, int X, int W, int SL, int ST, int NT, int NL, bool STORE, int SIG>
 __global__ void __launch_bounds__((W + 1 + NL) * 32, 1)
 plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = LayoutT<T, A, K, X, W, SL, ST, NT>;
@@ -189,7 +190,10 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const long long ntiles = (long long)prm.ntiles;
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
-    const Tables<T, A>& tb = prm.tab;
+    // SIG != 0: the signature's tables are compile-time constants (plr_constsig.cuh)
+    constexpr Tables<T, A> kTab = const_tables<T, A>(SIG, X, W);
+    static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
+    const Tables<T, A>& tb = SIG != 0 ? kTab : prm.tab;
 
     if (tid == 0) {
         for (int s = 0; s < SL; s++) { mbar_init(&full_L[s], 1); mbar_init(&empty_L[s], NC); }
@@ -410,7 +414,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             Gp[q] = sG[slot * kMaxK + q];
             Win[q] = sPw[(slot * W + warp) * K + q];
         }
-        matvec_acc<A, K>(Win, tb.Twin[warp], Gp);              // warp carry-in
+        matvec_acc<A, K>(Win, prm.tab.Twin[warp], Gp);         // warp carry-in (runtime index: parameter tables)
         tmem_wait_ld();
 #pragma unroll
         for (int q = 0; q < K; q++) {                           // thread carry-in

@@ -24,6 +24,7 @@ struct LaunchArgs {
     const void* lane_T;
     unsigned long long* stats = nullptr;
     int grid;
+    int sig = 0;                        // compile-time signature id (plr_constsig.cuh), 0 = runtime tables
     bool store;
     cudaStream_t stream;
     int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel

@@ -20,6 +20,7 @@
 #include <cstring>
 #include <vector>
 
+#include "plr_constsig.cuh"
 #include "plr_internal.h"
 
 namespace plr {
@@ -157,6 +158,17 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         else if (nnz == 1 && ones == 1) pt.cls = PLR_CLASS_PERM;
         else pt.cls = PLR_CLASS_POLY;
         pt.decay_flag = 0;
+        // compile-time signature kernels for the integer rows of Table 1
+        // (P:96-104), a0 = 1, p = 0 (plr_constsig.cuh)
+        pt.sig_id = 0;
+        if (p == 0 && pt.a_u[0] == 1u) {
+            for (int sig = kSigPrefix; sig <= kSigOrder3; sig++) {
+                if (const_sig_k(sig) != k) continue;
+                bool eq = true;
+                for (int j = 0; j < k; j++) eq = eq && c[j] == const_sig_c(sig, j);
+                if (eq) pt.sig_id = sig;
+            }
+        }
     } else {
         double c[kMaxK] = {0}, al[kMaxP + 1] = {0};
         for (int j = 0; j <= p; j++) al[j] = pt.a_d[j] = (double)(float)a[j];

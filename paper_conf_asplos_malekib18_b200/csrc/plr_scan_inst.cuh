@@ -5,6 +5,7 @@
 #include "plr_kernels.cuh"
 #include "plr_kernels_tmem.cuh"
 #include "plr_launch.h"
+#include <type_traits>
 
 namespace plr {
 namespace inst {
@@ -39,7 +40,7 @@ namespace inst {
 #ifndef PLR_TM_X
 #define PLR_TM_X 15
 #define PLR_TM_W 16
-#define PLR_TM_NL 2
+#define PLR_TM_NL 3
 #define PLR_TM_SL 3
 #define PLR_TM_ST 3
 #endif
@@ -66,7 +67,7 @@ struct TmCfg {
     static constexpr int NT = NT0 > PLR_TM_NTMAX ? PLR_TM_NTMAX : NT0;
 };
 
-template <typename T, typename A, class C, int K, int P, bool STORE>
+template <typename T, typename A, class C, int K, int P, bool STORE, int SIG = 0>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     constexpr bool tmem = PLR_GEN_TMEM && !C::DEC;
     size_t smem;
@@ -74,7 +75,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     void (*kern)(const ScanParams<T, A>);
     if constexpr (tmem) {
         using TC = TmCfg<T, A, K>;
-        kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, STORE>;
+        kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, STORE, SIG>;
         smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
         threads = (TC::W + 1 + TC::NL) * 32;
     } else {
@@ -114,8 +115,28 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     return cudaGetLastError();
 }
 
+// compile-time signature kernels (int32 ring, p = 0, TMEM kernel only)
+template <typename T, typename A, class C, int K, int SIG>
+cudaError_t launch_sig(const Tables<T, A>& tab, const LaunchArgs& la) {
+    return la.store ? launch_kps<T, A, C, K, 0, true, SIG>(tab, la) : launch_kps<T, A, C, K, 0, false, SIG>(tab, la);
+}
+
 template <typename T, typename A, class C, int K>
 cudaError_t launch_k(const Tables<T, A>& tab, const LaunchArgs& la, int p) {
+    if constexpr (std::is_same<T, uint32_t>::value && std::is_same<A, uint32_t>::value && PLR_GEN_TMEM && !C::DEC) {
+        if (la.sig != 0 && p == 0) {
+            if constexpr (K == 1) { if (la.sig == kSigPrefix) return launch_sig<T, A, C, 1, kSigPrefix>(tab, la); }
+            if constexpr (K == 2) {
+                if (la.sig == kSigTuple2) return launch_sig<T, A, C, 2, kSigTuple2>(tab, la);
+                if (la.sig == kSigOrder2) return launch_sig<T, A, C, 2, kSigOrder2>(tab, la);
+            }
+            if constexpr (K == 3) {
+                if (la.sig == kSigTuple3) return launch_sig<T, A, C, 3, kSigTuple3>(tab, la);
+                if (la.sig == kSigOrder3) return launch_sig<T, A, C, 3, kSigOrder3>(tab, la);
+            }
+            return cudaErrorInvalidValue;
+        }
+    }
     switch (p) {
         case 0: return la.store ? launch_kps<T, A, C, K, 0, true>(tab, la) : launch_kps<T, A, C, K, 0, false>(tab, la);
         case 1: return la.store ? launch_kps<T, A, C, K, 1, true>(tab, la) : launch_kps<T, A, C, K, 1, false>(tab, la);

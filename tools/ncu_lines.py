@@ -1,0 +1,31 @@
+"""Per-source-line warp-stall samples of an ncu capture (cuda,sass view).
+Usage: python tools/ncu_lines.py rep.ncu-rep [top]"""
+import csv
+import io
+import subprocess
+import sys
+
+rep = sys.argv[1]
+top = int(sys.argv[2]) if len(sys.argv) > 2 else 25
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+                     capture_output=True, text=True).stdout
+agg = {}
+cur = None
+fname = "?"
+for row in csv.reader(io.StringIO(out)):
+    if len(row) == 2 and row[0] == "File Path":
+        fname = row[1].split("/")[-1]
+        continue
+    if len(row) < 5 or row[0] == "Line No":
+        continue
+    if row[0]:
+        cur = (fname, row[0], row[1].strip()[:90])
+    try:
+        s = int(row[4])
+    except ValueError:
+        continue
+    if cur:
+        agg[cur] = agg.get(cur, 0) + s
+tot = sum(agg.values()) or 1
+for (f, ln, src), s in sorted(agg.items(), key=lambda kv: -kv[1])[:top]:
+    print("%5.1f%%  %s:%s  %s" % (100.0 * s / tot, f, ln, src))
