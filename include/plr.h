@@ -94,6 +94,7 @@ typedef struct {
                                   compile-time constants (the generator's per-signature
                                   code); 0: tables read from the
                                   kernel parameters                                   */
+    int tiles_per_unit;        /* G: consecutive tiles per ticket / status record / look-back */
 } plr_plan_info;
 
 /* Create a plan.  a[0..p] = (a0, a-1, ..., a-p) (p = feed-forward order, so

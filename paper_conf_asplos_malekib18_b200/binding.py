@@ -57,7 +57,8 @@ class PlanInfo(ctypes.Structure):
     _fields_ = [("p", _I), ("k", _I), ("dtype", _I), ("cls", _I), ("elems_per_thread", _I),
                 ("threads_per_cta", _I), ("tile_elems", _I), ("stages", _I), ("decay_len", ctypes.c_int64),
                 ("fixup_len", ctypes.c_int64), ("n_max", _S), ("scratch_bytes", _S), ("ctas_per_sm", _I),
-                ("num_sms", _I), ("const_sig", _I)]
+                ("num_sms", _I), ("const_sig", _I),
+                ("tiles_per_unit", _I)]
 
 
 class PLRError(RuntimeError):

@@ -214,6 +214,8 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     if (n > plan->n_max) return fail(PLR_ERR_SIZE, "n exceeds the plan's n_max");
     const uint64_t m = (uint64_t)plan->pt.geo.tile();
     const uint64_t ntiles = (n + m - 1) / m;
+    const uint64_t G = (uint64_t)plan->pt.geo.G;            // tiles per ticket (look-back unit)
+    const uint64_t nunits = (ntiles + G - 1) / G;
     if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
         CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, stream), "status reset");
         CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, 8, stream), "ticket reset");
@@ -222,7 +224,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         plan->dirty = false;
     }
     plan->epoch++;
-    const uint64_t grid = std::min<uint64_t>(ntiles, (uint64_t)plan->num_sms * plan->ctas_per_sm);
+    const uint64_t grid = std::min<uint64_t>(nunits, (uint64_t)plan->num_sms * plan->ctas_per_sm);
     LaunchArgs la;
     la.x = x; la.y = y; la.n = n; la.ntiles = ntiles;
     la.ticket_base = plan->ticket_base;
@@ -243,7 +245,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         plan->dirty = true;
         return cuda_fail(e, "scan kernel launch");
     }
-    plan->ticket_base += ntiles + grid;   // each CTA makes exactly one failing grab
+    plan->ticket_base += nunits + grid;   // each CTA makes exactly one failing grab
     return PLR_OK;
 }
 
@@ -405,6 +407,7 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->ctas_per_sm = plan->ctas_per_sm;
     info->num_sms = plan->num_sms;
     info->const_sig = plan->sig_kernel ? plan->pt.sig_id : 0;
+    info->tiles_per_unit = plan->pt.geo.G;
     return PLR_OK;
 }
 

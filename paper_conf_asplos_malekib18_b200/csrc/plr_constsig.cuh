@@ -84,8 +84,9 @@ PLR_HD constexpr CMat const_sig_companion(int sig) {
 }
 
 // Tables<uint32_t, uint32_t> of signature `sig` for the tile geometry (X, W)
+// and look-back unit of G tiles
 template <typename T, typename A>
-PLR_HD constexpr Tables<T, A> const_tables(int sig, int X, int W) {
+PLR_HD constexpr Tables<T, A> const_tables(int sig, int X, int W, int G) {
     Tables<T, A> t{};
     if constexpr (sizeof(T) == 4 && sizeof(A) == 4 && T(-1) > T(0)) {   // uint32 ring only
         if (sig == 0) return t;
@@ -118,6 +119,13 @@ PLR_HD constexpr Tables<T, A> const_tables(int sig, int X, int W) {
         }
         P = cmat_pow(M, m);
         for (int e = 0; e < kMaxK * kMaxK; e++) t.Tm[e] = P.v[e];
+        CMat Gn{};
+        for (int i = 0; i < kMaxK; i++) Gn.v[i * kMaxK + i] = 1u;
+        for (int g = 0; g < kMaxG; g++) {
+            for (int e = 0; e < kMaxK * kMaxK; e++) t.Tsub[g][e] = Gn.v[e];
+            Gn = cmat_mul(Gn, P);
+        }
+        P = cmat_pow(M, m * (unsigned long long)G);          // look-back unit U = G m
         for (int s = 0; s < 9; s++) {
             for (int e = 0; e < kMaxK * kMaxK; e++) t.Tpow[s][e] = P.v[e];
             P = cmat_mul(P, P);

@@ -6,9 +6,9 @@ namespace plr {
 Geometry class_geometry(bool decay) {
     // x elements per thread (odd: conflict-free strided smem access) and W
     // compute warps per config; the ring depth is reported by scan_stages()
-    if (decay) return Geometry{inst::CfgDec::X, inst::CfgDec::W, inst::CfgDec::S};
-    if (PLR_GEN_TMEM) return Geometry{PLR_TM_X, PLR_TM_W, PLR_TM_SL};
-    return Geometry{inst::CfgGen::X, inst::CfgGen::W, inst::CfgGen::S};
+    if (decay) return Geometry{inst::CfgDec::X, inst::CfgDec::W, inst::CfgDec::S, 1};
+    if (PLR_GEN_TMEM) return Geometry{PLR_TM_X, PLR_TM_W, PLR_TM_SL, PLR_TM_G};
+    return Geometry{inst::CfgGen::X, inst::CfgGen::W, inst::CfgGen::S, 1};
 }
 
 int scan_stages(const PlanTables& pt) {

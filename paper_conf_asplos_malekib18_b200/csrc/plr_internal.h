@@ -22,8 +22,12 @@ constexpr int kStatusMaxBytes = 128; // bytes per status slot the plan allocates
 constexpr int kAug = 8;             // augmented state slots: x_{-4..-1}, y_{-4..-1}
 constexpr int kTPL = 8;             // look-back: tiles per lane in a wide window (2^3)
 
+constexpr int kMaxG = 8;            // tiles per look-back unit (ticket)
+
+// G consecutive tiles form one look-back unit: one ticket, one status record
+// and one look-back per unit (the generic TMEM kernel; G = 1 elsewhere).
 struct Geometry {
-    int X, W, S;
+    int X, W, S, G;
     int tile() const { return 32 * W * X; }
 };
 
@@ -42,7 +46,8 @@ struct Tables {
     A Tblk[4][kMaxK * kMaxK];            // T(32 X * 2^s)       warp-aggregate scan
     A Twin[kMaxW][kMaxK * kMaxK];        // T(32 X * w)         warp carry-in
     A Tm[kMaxK * kMaxK];                 // T(m)                inclusive = agg + T(m) G
-    A Tpow[9][kMaxK * kMaxK];            // T(m * 2^s), s <= 8  look-back folds and skips
+    A Tpow[9][kMaxK * kMaxK];            // T(U * 2^s), s <= 8  look-back folds and skips (unit U = G m)
+    A Tsub[kMaxG][kMaxK * kMaxK];        // T(g m), g < G       tile carries inside a unit
 };
 
 template <typename T, typename A>

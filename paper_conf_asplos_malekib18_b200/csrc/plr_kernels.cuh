@@ -270,6 +270,24 @@ __device__ __forceinline__ int classify_status(const unsigned long long (&w)[Sta
 }
 
 
+// look-back debug counters (PLR_STATS=1): summed per warp in registers,
+// flushed with one atomic per counter when the warp exits
+// in shared memory (kLbStatWords per look-back warp), flushed with one atomic
+// per counter when the warp exits; registers stay free for the look-back
+constexpr int kLbStatWords = 9;
+constexpr int kMaxNL = 4;                              // look-back warps per CTA
+struct LbStats {
+    unsigned long long* v;                             // this warp's shared counters
+    __device__ void init(int lane) const {
+        if (lane == 0)
+            for (int i = 0; i < kLbStatWords; i++) v[i] = 0;
+    }
+    __device__ void flush(unsigned long long* dst, int lane) const {
+        if (dst != nullptr && lane == 0)
+            for (int i = 0; i < kLbStatWords; i++) atomicAdd(&dst[i], v[i]);
+    }
+};
+
 // Generic look-back: fold the tiles j-1, j-2, ...
 // nearest first, G_{j-1} = sum_d T(d m) v_{j-1-d}, v = aggregate for "P"
 // tiles and the inclusive carry of the first "I" tile.  Each poll reads a
@@ -279,7 +297,7 @@ __device__ __forceinline__ int classify_status(const unsigned long long (&w)[Sta
 template <typename T, typename A, int K, bool DEC>
 __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, const Tables<T, A>& tb, long long j,
                                                  int lane, uint32_t tagA, uint32_t tagI, A (&Gp)[K],
-                                                 long long c_start = 0, long long c_agg = 0) {
+                                                 const LbStats& lbs, long long c_start = 0, long long c_agg = 0) {
     long long c_wait = 0;
     // tiles per lane of a full window: 8 for small records, 4 when a record
     // has more than 2 words (keeps the window's registers in check)
@@ -400,17 +418,16 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
             ns = ns < 512 ? 2 * ns : ns;
         }
     }
-    if (prm.stats != nullptr && lane == 0) {
-        atomicAdd(&prm.stats[0], 1ull);                // look-backs
-        atomicAdd(&prm.stats[1], n_win);               // window polls
-        atomicAdd(&prm.stats[2], n_wait);              // polls that folded nothing
-        atomicAdd(&prm.stats[3], (unsigned long long)(o + 1));  // depth folded (approx.)
-        atomicAdd(&prm.stats[4], (unsigned long long)(c_agg - c_start));    // cycles waiting own A
-        atomicAdd(&prm.stats[5], (unsigned long long)(clock64() - c_agg));  // cycles looking back
-        atomicAdd(&prm.stats[6], (unsigned long long)c_wait);               // of which sleeping
-        atomicAdd(&prm.stats[7], (unsigned long long)c_load);               // loading + classifying windows
-        atomicAdd(&prm.stats[8], (unsigned long long)c_fold);               // folding
-
+    if (prm.stats != nullptr && lane == 0) {           // debug counters (shared, per warp)
+        lbs.v[0] += 1;                                 // look-backs
+        lbs.v[1] += n_win;                             // window polls
+        lbs.v[2] += n_wait;                            // polls that folded nothing
+        lbs.v[3] += (unsigned long long)(o + 1);       // depth folded (approx.)
+        lbs.v[4] += (unsigned long long)(c_agg - c_start);    // cycles waiting for the own aggregate
+        lbs.v[5] += (unsigned long long)(clock64() - c_agg);  // cycles looking back
+        lbs.v[6] += (unsigned long long)c_wait;               // of which sleeping
+        lbs.v[7] += (unsigned long long)c_load;               // loading + classifying windows
+        lbs.v[8] += (unsigned long long)c_fold;               // folding
     }
 #pragma unroll
     for (int q = 0; q < K; q++) Gp[q] = acc[q];
@@ -433,7 +450,8 @@ struct Layout {
     // bars: full[S], done[S], agg[NS], carry[NS]
     static constexpr size_t off_tile = off_bar + (2 * S + 2 * NS) * 8;               // tile_of[S]
     static constexpr size_t off_aggtile = off_tile + S * 8;                           // agg_tile[NS]
-    static constexpr size_t bytes = off_aggtile + NS * 8;
+    static constexpr size_t off_lbstat = off_aggtile + NS * 8;                        // [kMaxNL][kLbStatWords]
+    static constexpr size_t bytes = off_lbstat + kMaxNL * kLbStatWords * 8;
 };
 
 // ------------------------------------------------------ the scan kernel ----
@@ -542,6 +560,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // waiting for the tile's own aggregate, which the compute warps publish.
     if (warp > W) {
         const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
+        static_assert(NL <= kMaxNL, "look-back warps");
+        const LbStats lbs{reinterpret_cast<unsigned long long*>(smem + L::off_lbstat) + (warp - W - 1) * kLbStatWords};
+        lbs.init(lane);
         for (int it = warp - (W + 1);; it += NL) {     // NL look-back warps take turns
             const int s = it % S;
             const int slot = it % NS;
@@ -587,7 +608,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     mbar_wait(&agg_bar[nx % NS], (uint32_t)((nx / NS) & 1));
                 }
                 const long long c_agg = clock64();
-                lookback_generic<T, A, K, DEC>(prm, tb, j, lane, tagA, tagI, Gp, c_start, c_agg);
+                lookback_generic<T, A, K, DEC>(prm, tb, j, lane, tagA, tagI, Gp, lbs, c_start, c_agg);
             }
             // the tile's own aggregate (phase A) is needed for its inclusive carry
             if (j == 0 || DEC) mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
@@ -608,6 +629,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 if (lane == 0) mbar_arrive(&carry_bar[slot]);
             }
         }
+        lbs.flush(prm.stats, lane);
         return;
     }
 

@@ -140,16 +140,20 @@ struct LayoutT {
     static constexpr size_t off_bar = (off_wagg + (size_t)NT * W * kMaxK * sizeof(A) + 15) & ~(size_t)15;
     // bars: full_L[SL], empty_L[SL], full_T[ST], empty_T[ST], agg[NT], carry[NT]
     static constexpr size_t off_ids = off_bar + (size_t)(2 * SL + 2 * ST + 2 * NT) * 8;
-    // ids: tile_of[SL], store_tile[ST], slot_tile[NT] (long long), tmem base (u32)
+    // ids: tile_of[SL], store_tile[ST], slot_tile[NT] (long long), tmem base (u32),
+    // stop position (pipeline index of the compute warps' stop marker)
     static constexpr size_t off_tmem = off_ids + (size_t)(SL + ST + NT) * 8;
-    static constexpr size_t bytes = off_tmem + 16;
+    static constexpr size_t off_stop = off_tmem + 4;
+    static constexpr size_t off_lbstat = off_tmem + 16;                         // [kMaxNL][kLbStatWords]
+    static constexpr size_t bytes = off_lbstat + kMaxNL * kLbStatWords * 8;
 };
 
 // TMEM columns per warp per parked tile: X chunk values + K carries (A words)
 template <typename A, int K, int X>
 struct TmemCols { static constexpr int CW = X + K * AWords<A>::N; };
 
-template <typename T, typename A, int K, int P, int X, int W, int SL, int ST, int NT, int NL, bool STORE, int SIG>
+template <typename T, typename A, int K, int P, int X, int W, int SL, int ST, int NT, int NL, int G, bool STORE,
+          int SIG>
 __global__ void __launch_bounds__((W + 1 + NL) * 32, 1)
 plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = LayoutT<T, A, K, X, W, SL, ST, NT>;
@@ -165,6 +169,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     static_assert(X >= K && X <= kMaxX && (X & 1), "X must be odd and >= K");
     static_assert(NT >= 2 && NT * WQ * CW <= 512, "TMEM columns");
     static_assert(P <= kHalo, "halo");
+    static_assert(G >= 1 && G <= kMaxG && G + 1 <= NT, "look-back unit of G tiles needs G+1 parked tiles");
     constexpr bool DEC = false;
 
     extern __shared__ __align__(128) unsigned char smem[];
@@ -184,6 +189,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     long long* store_tile = tile_of + SL;
     long long* slot_tile = store_tile + ST;
     uint32_t* tmem_base_p = reinterpret_cast<uint32_t*>(smem + L::off_tmem);
+    volatile int* stop_pos = reinterpret_cast<volatile int*>(smem + L::off_stop);
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -191,7 +197,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
     // SIG != 0: the signature's tables are compile-time constants (plr_constsig.cuh)
-    constexpr Tables<T, A> kTab = const_tables<T, A>(SIG, X, W);
+    constexpr Tables<T, A> kTab = const_tables<T, A>(SIG, X, W, G);
     static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
     const Tables<T, A>& tb = SIG != 0 ? kTab : prm.tab;
 
@@ -199,6 +205,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         for (int s = 0; s < SL; s++) { mbar_init(&full_L[s], 1); mbar_init(&empty_L[s], NC); }
         for (int s = 0; s < ST; s++) { mbar_init(&full_T[s], NC); mbar_init(&empty_T[s], 1); }
         for (int s = 0; s < NT; s++) { mbar_init(&agg_bar[s], 1); mbar_init(&carry_bar[s], 1); }
+        *stop_pos = 1 << 30;
         fence_mbar_init();
     }
     if (warp == 0) tmem_alloc(tmem_base_p, 512);
@@ -211,12 +218,22 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     if (warp == W) {
         const uint64_t pol = policy_evict_first();
         if (lane == 0) {                                            // loader
+            long long unit = 0;
             for (int f = 0;; f++) {
                 const int s = f % SL;
                 if (f >= SL) mbar_wait(&empty_L[s], (uint32_t)(((f / SL) - 1) & 1));
-                const long long j = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
+                // one ticket per look-back unit of G consecutive tiles
+                if (f % G == 0) unit = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
+                long long j = unit * G + f % G;
+                if (j >= ntiles) j = ntiles;
                 tile_of[s] = j;
-                if (j >= ntiles) { mbar_arrive(&full_L[s]); break; }
+                if (j >= ntiles) {
+                    // the CTA that ends inside the last (partial) unit still makes
+                    // its one failing grab: the host counts nunits + grid tickets
+                    if (f % G != 0) atomicAdd(prm.ticket, 1ull);
+                    mbar_arrive(&full_L[s]);
+                    break;
+                }
                 if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_L[s]); continue; }
                 T* st = lstage + (size_t)s * SWL;
                 if (j == 0) {
@@ -262,32 +279,84 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     }
 
     // ===================================================== look-back warps ==
+    // Per look-back unit of G consecutive tiles (one ticket): fold the tile
+    // aggregates into the unit's local inclusive prefixes L_g = A_g + T(m)
+    // L_{g-1}, publish the unit aggregate, look back over the preceding units
+    // for the carry G_{J-1} entering the unit, hand
+    // every tile its carry-in L_{g-1} + T(g m) G_{J-1} and publish the unit's
+    // inclusive carry L_{G-1} + T(G m) G_{J-1}.
     if (warp > W) {
         const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
-        for (int it = warp - (W + 1);; it += NL) {
-            const int slot = it % NT;
-            mbar_wait(&agg_bar[slot], (uint32_t)((it / NT) & 1));
-            const long long j = slot_tile[slot];
-            if (j >= ntiles) break;
-            A Gp[K];
-            if (j == 0) {
+        static_assert(NL <= kMaxNL, "look-back warps");
+        const LbStats lbs{reinterpret_cast<unsigned long long*>(smem + L::off_lbstat) + (warp - W - 1) * kLbStatWords};
+        lbs.init(lane);
+        // wait for the aggregate of pipeline position p; false at the stop
+        auto wait_agg = [&](int p) -> bool {
+            const int slot = p % NT;
+            const uint32_t par = (uint32_t)((p / NT) & 1);
+            while (!mbar_try_wait(&agg_bar[slot], par))
+                if (*stop_pos <= p) return false;
+            return slot_tile[slot] < ntiles;
+        };
+        for (int u = warp - (W + 1);; u += NL) {               // NL look-back warps take turns
+            const long long c_start = clock64();
+            A Lp[G][K];                                        // local inclusive prefixes
+            int cnt = 0;
+#pragma unroll
+            for (int g = 0; g < G; g++) {
+                if (g == cnt && wait_agg(u * G + g)) {
+                    const int slot = (u * G + g) % NT;
+#pragma unroll
+                    for (int q = 0; q < K; q++) Lp[g][q] = sAt[slot * kMaxK + q];
+                    if (g > 0) matvec_acc<A, K>(Lp[g], tb.Tm, Lp[g - 1]);
+                    cnt++;
+                }
+            }
+            if (cnt == 0) break;
+            const long long J = slot_tile[(u * G) % NT] / G;   // unit index
+            A Gp[K];                                           // G_{J-1}: carries entering the unit
+            if (J == 0) {
 #pragma unroll
                 for (int q = 0; q < K; q++) Gp[q] = prm.y_hist != nullptr ? A(prm.y_hist[K - 1 - q]) : A(0);
             } else {
-                lookback_generic<T, A, K, DEC>(prm, tb, j, lane, tagA, tagI, Gp);
-            }
-            if (lane == 0) {
+                // publish the unit aggregate at once, then look back
+                A Ag[K];
 #pragma unroll
-                for (int q = 0; q < K; q++) sG[slot * kMaxK + q] = Gp[q];
-            }
-            A G[K];
+                for (int q = 0; q < K; q++) Ag[q] = Lp[G - 1][q];
 #pragma unroll
-            for (int q = 0; q < K; q++) G[q] = sAt[slot * kMaxK + q];
-            matvec_acc<A, K>(G, tb.Tm, Gp);                       // G_j = A_j + T(m) G_{j-1}
+                for (int g = 0; g + 1 < G; g++)
+                    if (g + 1 == cnt)
+#pragma unroll
+                        for (int q = 0; q < K; q++) Ag[q] = Lp[g][q];
+                publish_status<A, K, DEC>(prm.status, prm.status_mask, J, Ag, tagA, lane);
+                // stats: "agg" = idle until the unit's aggregate, "lb" = look-back
+                lookback_generic<T, A, K, DEC>(prm, tb, J, lane, tagA, tagI, Gp, lbs, c_start, clock64());
+            }
+#pragma unroll
+            for (int g = 0; g < G; g++) {
+                if (g < cnt) {
+                    const int slot = (u * G + g) % NT;
+                    A C[K];                                    // carry entering tile g
+#pragma unroll
+                    for (int q = 0; q < K; q++) C[q] = g == 0 ? A(0) : Lp[g > 0 ? g - 1 : 0][q];
+                    matvec_acc<A, K>(C, tb.Tsub[g], Gp);
+                    if (lane == 0) {
+#pragma unroll
+                        for (int q = 0; q < K; q++) sG[slot * kMaxK + q] = C[q];
+                    }
+                }
+            }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&carry_bar[slot]);
-            publish_status<A, K, DEC>(prm.status, prm.status_mask, j, G, tagI, lane);
+            if (lane == 0)
+                for (int g = 0; g < cnt; g++) mbar_arrive(&carry_bar[(u * G + g) % NT]);
+            if (cnt < G) break;                                // the CTA's last (partial) unit
+            A Gi[K];
+#pragma unroll
+            for (int q = 0; q < K; q++) Gi[q] = Lp[G - 1][q];
+            matvec_acc<A, K>(Gi, tb.Tpow[0], Gp);              // G_J = L_{G-1} + T(G m) G_{J-1}
+            publish_status<A, K, DEC>(prm.status, prm.status_mask, J, Gi, tagI, lane);
         }
+        lbs.flush(prm.stats, lane);
         return;
     }
 
@@ -304,7 +373,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         mbar_wait(&full_L[s], (uint32_t)((it / SL) & 1));
         const long long j = tile_of[s];
         if (j >= ntiles) {
-            if (tid == 0) { slot_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
+            if (tid == 0) { slot_tile[slot] = j; *stop_pos = it; mbar_arrive(&agg_bar[slot]); }
             return j;
         }
         const bool ragged = (j == ntiles - 1) && last_ragged;
@@ -390,10 +459,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (lane == 0) sPw[(slot * W + warp) * K + q] = warp == 0 ? A(0) : pw;
             if (tid == 0) sAt[slot * kMaxK + q] = At[q];
         }
-        // publish the aggregate at once; tile 0's inclusive carry
-        // is published by its look-back warp
-        if (warp == 0 && j > 0)
-            publish_status<A, K, DEC>(prm.status, prm.status_mask, j, At, 2u * prm.epoch, lane);
+        // the look-back warp folds the tile aggregate into its unit's
         tmem_wait_st();
         __syncwarp();
         if (tid == 0) { slot_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
@@ -483,10 +549,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         if (tid == 0) store_tile[sT] = ntiles;
         mbar_arrive(&full_T[sT]);
     }
-    for (int it = na + 1; it < na + NL; it++) {
-        // every earlier phase of these slots has been consumed (all carries arrived)
-        if (tid == 0) { slot_tile[it % NT] = ntiles; mbar_arrive(&agg_bar[it % NT]); }
-    }
+    // look-back warps waiting beyond the stop see *stop_pos (set by phase A)
     tc_fence_before();
     named_sync(1, NC);
     if (warp == 0) {

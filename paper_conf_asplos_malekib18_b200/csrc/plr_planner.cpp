@@ -96,7 +96,9 @@ void fill_tables(const Mat<R>& M, int k, Geometry geo, Tables<T, A>* tb, A* lane
     for (int s = 0; s < 4; s++) store_mat(mpow(M, (32 * X) << s), tb->Tblk[s], cvtA);
     for (int w = 0; w < kMaxW; w++) store_mat(mpow(M, 32 * X * (uint64_t)w), tb->Twin[w], cvtA);
     store_mat(mpow(M, m), tb->Tm, cvtA);
-    for (int s = 0; s < 9; s++) store_mat(mpow(M, m << s), tb->Tpow[s], cvtA);
+    const uint64_t U = m * (uint64_t)geo.G;                  // look-back unit
+    for (int s = 0; s < 9; s++) store_mat(mpow(M, U << s), tb->Tpow[s], cvtA);
+    for (int g = 0; g < kMaxG; g++) store_mat(mpow(M, m * (uint64_t)g), tb->Tsub[g], cvtA);
     for (int l = 0; l < 32; l++) {
         Mat<R> Tl = mpow(M, X * (uint64_t)l);
         for (int q = 0; q < k; q++)
@@ -133,7 +135,10 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         }
         if ((float)a[p] == 0.0f || (float)b[k - 1] == 0.0f) { *why = "last coefficient rounds to 0 in fp32"; return PLR_ERR_SIGNATURE; }
     }
-    if (geo.X < k || geo.X > kMaxX || geo.W > kMaxW || (geo.W & (geo.W - 1))) { *why = "bad geometry"; return PLR_ERR_INVALID_ARG; }
+    if (geo.X < k || geo.X > kMaxX || geo.W > kMaxW || (geo.W & (geo.W - 1)) || geo.G < 1 || geo.G > kMaxG) {
+        *why = "bad geometry";
+        return PLR_ERR_INVALID_ARG;
+    }
 
     PlanTables& pt = *out;
     std::memset(&pt, 0, sizeof(pt));

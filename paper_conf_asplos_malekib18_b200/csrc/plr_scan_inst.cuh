@@ -40,9 +40,12 @@ namespace inst {
 #ifndef PLR_TM_X
 #define PLR_TM_X 15
 #define PLR_TM_W 16
-#define PLR_TM_NL 3
+#define PLR_TM_NL 2
 #define PLR_TM_SL 3
 #define PLR_TM_ST 3
+#endif
+#ifndef PLR_TM_G
+#define PLR_TM_G 3          // tiles per look-back unit (one ticket, one look-back)
 #endif
 
 // S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
@@ -58,7 +61,7 @@ using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_G
 
 template <typename T, typename A, int K>
 struct TmCfg {
-    static constexpr int X = PLR_TM_X, W = PLR_TM_W, NL = PLR_TM_NL, SL = PLR_TM_SL, ST = PLR_TM_ST;
+    static constexpr int X = PLR_TM_X, W = PLR_TM_W, NL = PLR_TM_NL, SL = PLR_TM_SL, ST = PLR_TM_ST, G = PLR_TM_G;
     static constexpr int CW = dev::TmemCols<A, K, X>::CW;
 #ifndef PLR_TM_NTMAX
 #define PLR_TM_NTMAX 8
@@ -75,7 +78,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     void (*kern)(const ScanParams<T, A>);
     if constexpr (tmem) {
         using TC = TmCfg<T, A, K>;
-        kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, STORE, SIG>;
+        kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, TC::G, STORE, SIG>;
         smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
         threads = (TC::W + 1 + TC::NL) * 32;
     } else {
