@@ -251,8 +251,9 @@ def main():
                          "frac": round(achieved / hbm, 4),
                          "traffic": (traffic or {}).get("bytes_per_launch"),
                          "peak_source": "MEASURED_PEAKS.json hbm_gbs (%s)" % peaks_src,
-                         "kernel": "plr_scan_kernel (single pass), avg of %d launches, CUDA events on the launch stream"
-                                   % len(kern_ms),
+                         "kernel": "%s (single pass), avg of %d launches, CUDA events on the launch stream"
+                                   % (plans[WORKLOAD_SIGS[0]].kernel_name(), len(kern_ms)),
+                         "traffic_source": (traffic or {}).get("source"),
                          "kernel_ms": round(kern_avg, 4),
                          "algorithmic_bytes_per_launch": n * BYTES_PER_ELT},
             "gpu_launches": args.steps * len(WORKLOAD_SIGS) * (1 if world == 1 else 6),

@@ -95,6 +95,8 @@ typedef struct {
                                   code); 0: tables read from the
                                   kernel parameters                                   */
     int tiles_per_unit;        /* G: consecutive tiles per ticket / status record / look-back */
+    int kernel_kind;           /* scan kernel: 0 DECAY single-hop pipeline, 1 TMEM-parking,
+                                  2 L2 re-read (generic classes), 3 generic smem pipeline */
 } plr_plan_info;
 
 /* Create a plan.  a[0..p] = (a0, a-1, ..., a-p) (p = feed-forward order, so

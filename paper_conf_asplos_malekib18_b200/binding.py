@@ -58,7 +58,7 @@ class PlanInfo(ctypes.Structure):
                 ("threads_per_cta", _I), ("tile_elems", _I), ("stages", _I), ("decay_len", ctypes.c_int64),
                 ("fixup_len", ctypes.c_int64), ("n_max", _S), ("scratch_bytes", _S), ("ctas_per_sm", _I),
                 ("num_sms", _I), ("const_sig", _I),
-                ("tiles_per_unit", _I)]
+                ("tiles_per_unit", _I), ("kernel_kind", _I)]
 
 
 class PLRError(RuntimeError):
@@ -139,6 +139,12 @@ class Plan:
             self.close()
         except Exception:
             pass
+
+    KERNEL_NAMES = {0: "plr_scan_kernel (DECAY single-hop pipeline)", 1: "plr_scan_tmem_kernel (TMEM parking)",
+                    2: "plr_scan_rr_kernel (L2 re-read)", 3: "plr_scan_kernel (generic pipeline)"}
+
+    def kernel_name(self) -> str:
+        return self.KERNEL_NAMES.get(self.info["kernel_kind"], "?")
 
     @property
     def info(self) -> dict:

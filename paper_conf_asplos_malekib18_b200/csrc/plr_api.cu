@@ -318,14 +318,14 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     const char* why = "";
     // plan with the DECAY geometry; non-decaying plans are re-planned with
     // the generic kernel's geometry (the class is known after planning)
-    plr_status st = plan_tables(a, p, b, k, dtype, class_geometry(true), &plan->pt, &why);
+    plr_status st = plan_tables(a, p, b, k, dtype, class_geometry(true, k), &plan->pt, &why);
     // ablation (Fig. 10 analogue): PLR_FORCE_GENERIC=1 disables
     // the DECAY specialisation (single-hop look-back) for this plan
     const char* fg = std::getenv("PLR_FORCE_GENERIC");
     const bool force_generic = fg != nullptr && fg[0] == '1';
     if (st == PLR_OK && (!plan->pt.decay_flag || force_generic)) {
         plan_tables_free(&plan->pt);
-        st = plan_tables(a, p, b, k, dtype, class_geometry(false), &plan->pt, &why);
+        st = plan_tables(a, p, b, k, dtype, class_geometry(false, k), &plan->pt, &why);
         if (st == PLR_OK && force_generic) {
             plan->pt.decay_flag = 0;
             plan->pt.acc64 = dtype == PLR_FLOAT32 ? 1 : 0;   // generic float kernels accumulate in fp64
@@ -408,6 +408,7 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->num_sms = plan->num_sms;
     info->const_sig = plan->sig_kernel ? plan->pt.sig_id : 0;
     info->tiles_per_unit = plan->pt.geo.G;
+    info->kernel_kind = kernel_kind(plan->pt);
     return PLR_OK;
 }
 

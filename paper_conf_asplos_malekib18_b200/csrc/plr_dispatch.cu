@@ -3,17 +3,23 @@
 
 namespace plr {
 
-Geometry class_geometry(bool decay) {
+Geometry class_geometry(bool decay, int k) {
     // x elements per thread (odd: conflict-free strided smem access) and W
     // compute warps per config; the ring depth is reported by scan_stages()
     if (decay) return Geometry{inst::CfgDec::X, inst::CfgDec::W, inst::CfgDec::S, 1};
-    if (PLR_GEN_TMEM) return Geometry{PLR_TM_X, PLR_TM_W, PLR_TM_SL, PLR_TM_G};
+    switch (inst::gen_kind(k)) {
+        case 2: return Geometry{PLR_RR_X, PLR_RR_W, PLR_RR_SA + PLR_RR_SB, PLR_RR_G};
+        case 1: return Geometry{PLR_TM_X, PLR_TM_W, PLR_TM_SL + PLR_TM_ST, PLR_TM_G};
+    }
     return Geometry{inst::CfgGen::X, inst::CfgGen::W, inst::CfgGen::S, 1};
 }
 
-int scan_stages(const PlanTables& pt) {
-    if (pt.decay_flag) return inst::CfgDec::S;
-    return PLR_GEN_TMEM ? PLR_TM_SL : inst::CfgGen::S;
+int scan_stages(const PlanTables& pt) { return pt.geo.S; }
+
+int kernel_kind(const PlanTables& pt) {
+    if (pt.decay_flag) return 0;
+    const int kind = inst::gen_kind(pt.k);
+    return kind == 0 ? 3 : kind;
 }
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la) {

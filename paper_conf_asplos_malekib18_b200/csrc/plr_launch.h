@@ -31,7 +31,7 @@ struct LaunchArgs {
 };
 
 // Tile geometry of the DECAY / generic kernel configs.
-Geometry class_geometry(bool decay);
+Geometry class_geometry(bool decay, int k);
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm);
@@ -43,5 +43,7 @@ cudaError_t launch_scan_f64acc_dec(const Tables<float, double>& tab, const Launc
 cudaError_t launch_scan_f64acc_gen(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
 // ring depth of the config a plan launches with (plan info)
 int scan_stages(const PlanTables& pt);
+// plr_plan_info.kernel_kind of a plan
+int kernel_kind(const PlanTables& pt);
 
 }  // namespace plr

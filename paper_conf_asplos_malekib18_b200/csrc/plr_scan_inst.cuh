@@ -4,6 +4,7 @@
 #pragma once
 #include "plr_kernels.cuh"
 #include "plr_kernels_tmem.cuh"
+#include "plr_kernels_rr.cuh"
 #include "plr_launch.h"
 #include <type_traits>
 
@@ -31,11 +32,31 @@ namespace inst {
 #define PLR_GEN_W 16
 #define PLR_GEN_MINB 1
 #endif
-// generic classes use the TMEM-parking kernel (plr_kernels_tmem.cuh) unless
-// PLR_GEN_TMEM=0: X, W, NL as below, SL load + ST store stages, as many
-// parked tiles as fit in 512 TMEM columns (max 8)
-#ifndef PLR_GEN_TMEM
-#define PLR_GEN_TMEM 1
+// Kernel of the generic (non-decaying) classes, PLR_GEN_KIND:
+//   2 (default) re-read kernel (plr_kernels_rr.cuh): phase B re-reads x from
+//     L2 and recomputes from the true carry-in; lag NS-1 tiles
+//   1 TMEM-parking kernel (plr_kernels_tmem.cuh): chunk values of up to 8
+//     tiles parked in TMEM, phase B corrects them
+//   0 shared-memory pipeline kernel (plr_scan_kernel, S-stage ring)
+#ifndef PLR_GEN_KIND
+#define PLR_GEN_KIND 2
+#endif
+// first-order signatures (k = 1) use their own kernel kind: the TMEM kernel
+// reaches memcpy speed there (measured), the re-read kernel for k >= 2
+#ifndef PLR_K1_KIND
+#define PLR_K1_KIND 1
+#endif
+#define PLR_GEN_TMEM (PLR_GEN_KIND != 0)
+#ifndef PLR_RR_X
+#define PLR_RR_X 15
+#define PLR_RR_W 16
+#define PLR_RR_NL 2
+#define PLR_RR_SA 3         // phase-A (HBM) load stages
+#define PLR_RR_SB 4         // phase-B (L2 re-read + y store) stages
+#define PLR_RR_NS 7         // slots: phase B lags phase A by NS-1 tiles (L2 reuse distance)
+#endif
+#ifndef PLR_RR_G
+#define PLR_RR_G 3          // tiles per look-back unit (one ticket, one look-back)
 #endif
 #ifndef PLR_TM_X
 #define PLR_TM_X 15
@@ -47,6 +68,9 @@ namespace inst {
 #ifndef PLR_TM_G
 #define PLR_TM_G 3          // tiles per look-back unit (one ticket, one look-back)
 #endif
+
+// kernel kind of a non-decaying signature of order k (see PLR_GEN_KIND)
+constexpr int gen_kind(int k) { return k == 1 ? PLR_K1_KIND : PLR_GEN_KIND; }
 
 // S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
 // W compute warps (tile m = 32 W X)
@@ -72,11 +96,17 @@ struct TmCfg {
 
 template <typename T, typename A, class C, int K, int P, bool STORE, int SIG = 0>
 cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
-    constexpr bool tmem = PLR_GEN_TMEM && !C::DEC;
+    constexpr int kind = C::DEC ? 0 : gen_kind(K);
+    constexpr bool tmem = kind != 0;
     size_t smem;
     int threads;
     void (*kern)(const ScanParams<T, A>);
-    if constexpr (tmem) {
+    if constexpr (kind == 2) {
+        kern = &dev::plr_scan_rr_kernel<T, A, K, P, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS, PLR_RR_NL,
+                                         PLR_RR_G, STORE, SIG>;
+        smem = dev::LayoutR<T, A, K, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS>::bytes;
+        threads = (PLR_RR_W + 1 + PLR_RR_NL) * 32;
+    } else if constexpr (tmem) {
         using TC = TmCfg<T, A, K>;
         kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, TC::G, STORE, SIG>;
         smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
@@ -126,7 +156,7 @@ cudaError_t launch_sig(const Tables<T, A>& tab, const LaunchArgs& la) {
 
 template <typename T, typename A, class C, int K>
 cudaError_t launch_k(const Tables<T, A>& tab, const LaunchArgs& la, int p) {
-    if constexpr (std::is_same<T, uint32_t>::value && std::is_same<A, uint32_t>::value && PLR_GEN_TMEM && !C::DEC) {
+    if constexpr (std::is_same<T, uint32_t>::value && std::is_same<A, uint32_t>::value && gen_kind(K) != 0 && !C::DEC) {
         if (la.sig != 0 && p == 0) {
             if constexpr (K == 1) { if (la.sig == kSigPrefix) return launch_sig<T, A, C, 1, kSigPrefix>(tab, la); }
             if constexpr (K == 2) {

@@ -1,0 +1,13 @@
+# full GPU check: smoke, all -m gpu tests, per-signature timings, bench, ncu
+# (launch list of the bench command + full captures of the bench kernels)
+# usage: TAG=r01x bash tools/gpu_round.sh
+set -x
+TAG=${TAG:-r01}
+mkdir -p gpurun_out
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/${TAG}_smi.txt
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/${TAG}_smoke.log
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/${TAG}_pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/${TAG}_pytest_gpu.log
+timeout 300 python tools/time_sigs.py $((1<<30)) > gpurun_out/${TAG}_times.log 2>&1
+timeout 600 python bench.py > gpurun_out/${TAG}_bench.log 2>&1; echo "bench rc=$?" >> gpurun_out/${TAG}_bench.log
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 3 --warmup 3 > gpurun_out/${TAG}_bench_ncu.log 2>&1
+[ -z "$NONCU" ] && bash tools/ncu_profile.sh ${TAG} "${NCU_SIGS:-tuple2 tuple3}"

@@ -6,10 +6,11 @@ import subprocess
 import sys
 
 rep = sys.argv[1]
-top = int(sys.argv[2]) if len(sys.argv) > 2 else 25
+top = int(sys.argv[2]) if len(sys.argv) > 2 and sys.argv[2].isdigit() else 25
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                      capture_output=True, text=True).stdout
 agg = {}
+inst = {}
 cur = None
 fname = "?"
 for row in csv.reader(io.StringIO(out)):
@@ -24,8 +25,16 @@ for row in csv.reader(io.StringIO(out)):
         s = int(row[4])
     except ValueError:
         continue
+    try:
+        ie = int(row[7])
+    except (ValueError, IndexError):
+        ie = 0
     if cur:
         agg[cur] = agg.get(cur, 0) + s
+        inst[cur] = inst.get(cur, 0) + ie
 tot = sum(agg.values()) or 1
-for (f, ln, src), s in sorted(agg.items(), key=lambda kv: -kv[1])[:top]:
-    print("%5.1f%%  %s:%s  %s" % (100.0 * s / tot, f, ln, src))
+itot = sum(inst.values()) or 1
+key = (lambda kv: -inst[kv[0]]) if "--inst" in sys.argv else (lambda kv: -kv[1])
+print("stall%  inst%  line")
+for (f, ln, src), s in sorted(agg.items(), key=key)[:top]:
+    print("%5.1f%% %5.1f%%  %s:%s  %s" % (100.0 * s / tot, 100.0 * inst[(f, ln, src)] / itot, f, ln, src))
