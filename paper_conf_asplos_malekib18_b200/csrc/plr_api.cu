@@ -233,6 +233,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.status_mask = plan->status_slots - 1;
     la.epoch = plan->epoch;
     la.decay = plan->pt.decay_flag;
+    la.dec_mask = plan->pt.dec_mask;
     la.x_hist = x_hist; la.y_hist = y_hist; la.y_tail = y_tail;
     la.lane_T = plan->d_lane;
     la.stats = plan->d_stats;

@@ -62,6 +62,8 @@ struct ScanParams {
     uint32_t status_mask;                // 2^c - 1, 2^c >= ntiles
     uint32_t epoch;                      // tags 2*epoch (aggregate) / 2*epoch+1 (inclusive)
     int decay;                           // T(m) == 0 exactly: inclusive == aggregate
+    uint32_t dec_mask;                   // DECAY kernels: bit s < 5 = lane-scan step s has a non-negligible
+                                         // T(X 2^s); bit 5 = warp-aggregate level (T(32X d), d >= 1) non-negligible
     const T* x_hist;                     // p values x_{-p}..x_{-1} or null
     const T* y_hist;                     // k values y_{-k}..y_{-1} or null
     T* y_tail;                           // k slots y_{n-k}..y_{n-1} or null
@@ -80,6 +82,7 @@ struct PlanTables {
     int64_t fixup_len;
     int decay_flag;
     int acc64;                           // float: accumulate recurrence + carries in fp64
+    uint32_t dec_mask;                   // ScanParams::dec_mask of the tables the plan launches with
     double cond_bound;                   // eps32 * sum|a| * (sum|g|)^2 (float)
     int sig_id;                          // compile-time signature kernel (plr_constsig.cuh), 0 = none
     Tables<uint32_t, uint32_t> ti;       // int32 ring

@@ -57,8 +57,26 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
         : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
     return ok != 0;
 }
+// try_wait with a suspend-time hint: the waiting warp sleeps in hardware
+// until the phase completes (or the hint, in ns, expires) instead of spinning
+// through issue slots the working warps of its SM sub-partition need
+__device__ __forceinline__ bool mbar_try_wait_sleep(uint64_t* bar, uint32_t parity, uint32_t hint_ns) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity), "r"(hint_ns) : "memory");
+    return ok != 0;
+}
+#ifndef PLR_WAIT_HINT_NS
+#define PLR_WAIT_HINT_NS 0x989680u        // 10 ms: wake on completion
+#endif
+#ifndef PLR_POLL_HINT_NS
+#define PLR_POLL_HINT_NS 0u               // waits that also poll a stop flag (a hint measured slower)
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    while (!mbar_try_wait(bar, parity)) { }
+    while (!mbar_try_wait_sleep(bar, parity, PLR_WAIT_HINT_NS)) { }
 }
 // TMA 1D bulk copy global -> shared, completion on an mbarrier (UBLKCP).
 __device__ __forceinline__ void bulk_load(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar,
@@ -696,9 +714,11 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
         for (int q = 0; q < K; q++) v[q] = hist[q];             // local carry (l_{X-1}, ..., l_{X-K})
 
-        // a3: warp inclusive scan with T(X * 2^s)
+        // a3: warp inclusive scan with T(X * 2^s); DECAY skips the steps
+        // whose transfer matrix is negligible (dec_mask, uniform branch)
 #pragma unroll
         for (int s2 = 0; s2 < 5; s2++) {
+            if (DEC && !((prm.dec_mask >> s2) & 1u)) continue;
             A o[K];
 #pragma unroll
             for (int q = 0; q < K; q++) o[q] = shfl_up(v[q], 1 << s2);
@@ -719,6 +739,29 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
         for (int u = 0; u < X; u++) st[kHalo + tid * X + u] = lf[u];
 
+        // a4, DECAY with T(32X d) == 0 for d >= 1 (dec_mask bit 5 clear): the
+        // exclusive warp prefix is the previous warp's aggregate and the tile
+        // aggregate the last warp's ("only the first few warps")
+        if (DEC && !(prm.dec_mask & 32u)) {
+            if (lane == 0) {
+#pragma unroll
+                for (int q = 0; q < K; q++)
+                    sPw[(slot * W + warp) * K + q] = warp == 0 ? A(0) : wagg[(slot * W + warp - 1) * kMaxK + q];
+            }
+            if (tid == 0) {
+#pragma unroll
+                for (int q = 0; q < K; q++) sAt[slot * kMaxK + q] = wagg[(slot * W + W - 1) * kMaxK + q];
+            }
+            if (warp == 0) {
+                A At[K];
+#pragma unroll
+                for (int q = 0; q < K; q++) At[q] = wagg[(slot * W + W - 1) * kMaxK + q];
+                publish_status<A, K, DEC>(prm.status, prm.status_mask, j, At, 2u * prm.epoch + 1u, lane);
+            }
+            __syncwarp();
+            if (tid == 0) { agg_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
+            return j;
+        }
         // a4: scan of the W warp aggregates with T(32X * 2^s)
         A u_[K];
 #pragma unroll
@@ -766,7 +809,14 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             Gp[q] = sG[slot * kMaxK + q];
             Win[q] = sPw[(slot * W + warp) * K + q];
         }
-        matvec_acc<A, K>(Win, tb.Twin[warp], Gp);              // warp carry-in
+        if (DEC && !(prm.dec_mask & 32u)) {                    // T(32X w) == 0 for w >= 1
+            if (warp == 0) {
+#pragma unroll
+                for (int q = 0; q < K; q++) Win[q] = Gp[q];
+            }
+        } else {
+            matvec_acc<A, K>(Win, tb.Twin[warp], Gp);          // warp carry-in
+        }
 #pragma unroll
         for (int q = 0; q < K; q++) {                           // thread carry-in
             A acc = sE[(slot * K + q) * NC + tid];

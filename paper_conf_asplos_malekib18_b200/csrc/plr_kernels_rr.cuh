@@ -183,7 +183,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 const int slot = f % NS;
                 const uint32_t par = (uint32_t)((f / NS) & 1);
                 bool stop = false;
-                while (!mbar_try_wait(&agg_bar[slot], par))
+                while (!mbar_try_wait_sleep(&agg_bar[slot], par, PLR_POLL_HINT_NS))
                     if (*stop_pos <= f) { stop = true; break; }
                 const long long j = stop ? ntiles : slot_tile[slot];
                 if (j >= ntiles) break;
@@ -201,7 +201,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 // signalled through stop_pos (phase B never runs for it)
                 const uint32_t par = (uint32_t)((t / SB) & 1);
                 bool stop = false;
-                while (!mbar_try_wait(&yfull[sb], par))
+                while (!mbar_try_wait_sleep(&yfull[sb], par, PLR_POLL_HINT_NS))
                     if (*stop_pos <= t) { stop = true; break; }
                 if (stop) break;
                 const long long jt = store_tile[sb];
@@ -232,7 +232,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         auto wait_agg = [&](int p) -> bool {                     // false at the stop
             const int slot = p % NS;
             const uint32_t par = (uint32_t)((p / NS) & 1);
-            while (!mbar_try_wait(&agg_bar[slot], par))
+            while (!mbar_try_wait_sleep(&agg_bar[slot], par, PLR_POLL_HINT_NS))
                 if (*stop_pos <= p) return false;
             return slot_tile[slot] < ntiles;
         };

@@ -18,6 +18,7 @@ struct LaunchArgs {
     uint32_t status_mask;
     uint32_t epoch;
     int decay;
+    uint32_t dec_mask = 0x3f;
     const void* x_hist;
     const void* y_hist;
     void* y_tail;

@@ -106,6 +106,45 @@ void fill_tables(const Mat<R>& M, int k, Geometry geo, Tables<T, A>* tb, A* lane
     }
 }
 
+// DECAY tables whose entries are all below kCut are treated as exactly zero
+// (reading R17): a carry of magnitude <= 2^10 then moves an output
+// by <= 2^-50, nine decades under the 1e-4 tolerance.  The fp32 tables of
+// the warp-aggregate level (L >= 32X = 480 > L_dec) are already exactly zero.
+constexpr double kCut = 0x1p-60;
+
+template <typename A>
+bool negligible(const A* t) {
+    for (int e = 0; e < kMaxK * kMaxK; e++)
+        if (std::fabs((double)t[e]) > kCut) return false;
+    return true;
+}
+
+// ScanParams::dec_mask of a DECAY plan's tables; negligible tables are zeroed
+// so the kernels that still read them see the same values they skip.
+template <typename T, typename A>
+uint32_t decay_mask(Tables<T, A>* tb, A* lane, int k, Geometry geo) {
+    uint32_t mask = 0;
+    for (int s = 0; s < 5; s++) {
+        if (!negligible(tb->Twarp[s])) mask |= 1u << s;
+        else for (auto& e : tb->Twarp[s]) e = A(0);
+    }
+    bool blk = false;
+    for (int s = 0; s < 4; s++) blk = blk || !negligible(tb->Tblk[s]);
+    for (int w = 1; w < geo.W; w++) blk = blk || !negligible(tb->Twin[w]);
+    if (blk) {
+        mask |= 1u << 5;
+    } else {
+        for (int s = 0; s < 4; s++) for (auto& e : tb->Tblk[s]) e = A(0);
+        for (int w = 1; w < kMaxW; w++) for (auto& e : tb->Twin[w]) e = A(0);
+    }
+    for (int l = 0; l < 32; l++) {
+        double mx = 0.0;
+        for (int e = 0; e < k * k; e++) mx = std::fmax(mx, std::fabs((double)lane[e * 32 + l]));
+        if (mx <= kCut) for (int e = 0; e < k * k; e++) lane[e * 32 + l] = A(0);
+    }
+    return mask;
+}
+
 }  // namespace
 
 plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype dtype,
@@ -144,6 +183,7 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
     std::memset(&pt, 0, sizeof(pt));
     pt.p = p; pt.k = k; pt.dtype = dtype; pt.geo = geo;
     pt.decay_len = -1; pt.fixup_len = 0;
+    pt.dec_mask = 0x3fu;
     pt.fix_table = nullptr;
 
     if (dtype == PLR_INT32) {
@@ -217,6 +257,9 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         pt.cond_bound = std::ldexp(1.0, -24) * sa * sg * sg;
         pt.acc64 = (!decays || !(pt.cond_bound <= 1e-3)) ? 1 : 0;
         if (!pt.decay_flag) pt.acc64 = 1;      // multi-tile look-back kernels exist in fp64 accumulation only
+        pt.dec_mask = 0x3fu;
+        if (pt.decay_flag)                     // DECAY hierarchy: skip the negligible transfer matrices
+            pt.dec_mask = pt.acc64 ? decay_mask(&pt.td, pt.lane_d, k, geo) : decay_mask(&pt.tf, pt.lane_f, k, geo);
         if (decays) {
             pt.decay_len = last;
             // free response of the augmented state (x_{-4..-1}, y_{-4..-1})

@@ -138,6 +138,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     prm.status_mask = la.status_mask;
     prm.epoch = la.epoch;
     prm.decay = la.decay;
+    prm.dec_mask = la.dec_mask;
     prm.x_hist = static_cast<const T*>(la.x_hist);
     prm.y_hist = static_cast<const T*>(la.y_hist);
     prm.y_tail = static_cast<T*>(la.y_tail);

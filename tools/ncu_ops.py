@@ -1,26 +1,37 @@
-"""Per-opcode executed warp instructions per unit of work from an ncu capture.
-Usage: python tools/ncu_ops.py rep.ncu-rep units [top]"""
-import collections
+"""Dynamic SASS opcode mix of an ncu capture (source page, sass view):
+warp-level instructions executed per opcode, and per element of the launch.
+Usage: python tools/ncu_ops.py rep.ncu-rep [n_elements] [top]"""
 import csv
 import io
 import subprocess
 import sys
 
-rep, units = sys.argv[1], float(sys.argv[2])
+rep = sys.argv[1]
+n = float(sys.argv[2]) if len(sys.argv) > 2 else float(1 << 30)
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 30
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
-hdr = next(r for r in rows if r and r[0] == "Address")
-isrc, iex = hdr.index("Source"), hdr.index("Instructions Executed")
-ops = collections.Counter()
-for r in rows:
-    if len(r) <= iex or not r[iex].isdigit():
+hdr = rows[1]
+iS, iE, iT = hdr.index("Source"), hdr.index("Instructions Executed"), hdr.index("Thread Instructions Executed")
+agg, tagg = {}, {}
+for r in rows[2:]:
+    if len(r) <= iT:
         continue
-    toks = [t for t in r[isrc].split() if not t.startswith("@")]
-    if toks:
-        ops[toks[0].split(".")[0]] += int(r[iex])
-tot = sum(ops.values())
-print("total %.0f warp-inst per unit" % (tot / units))
-for op, c in ops.most_common(top):
-    print("%-10s %8.1f  %4.1f%%" % (op, c / units, 100.0 * c / tot))
+    src = r[iS].strip()
+    toks = src.split()
+    if not toks:
+        continue
+    op = toks[1] if toks[0].startswith("@") and len(toks) > 1 else toks[0]
+    op = op.split(".")[0].rstrip(";")
+    try:
+        e, t = int(r[iE]), int(r[iT])
+    except ValueError:
+        continue
+    agg[op] = agg.get(op, 0) + e
+    tagg[op] = tagg.get(op, 0) + t
+tot = sum(agg.values())
+print("total warp inst %.3e  = %.2f warp-inst/elt, %.1f thread-inst/elt (32x)" % (tot, tot / n, 32 * tot / n))
+print("%-10s %10s %8s %10s" % ("op", "warp-inst", "%", "thr/elt"))
+for op, e in sorted(agg.items(), key=lambda kv: -kv[1])[:top]:
+    print("%-10s %10.3e %7.1f%% %10.2f" % (op, e, 100.0 * e / tot, tagg[op] / n))
