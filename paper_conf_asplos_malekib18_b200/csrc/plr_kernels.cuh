@@ -119,6 +119,25 @@ __device__ __forceinline__ float mad(float a, float b, float c) { return __fmaf_
 __device__ __forceinline__ double mad(double a, double b, double c) { return __fma_rn(a, b, c); }
 
 
+// conversions between the data type and the accumulation type.  fp32 values
+// here come out of FTZ arithmetic (already flushed), so the plain cvt is used:
+// the compiler's default under -ftz adds a flushing FMUL / DSETP+FSEL per
+// conversion, one per element on the fp64-accumulation path.
+template <typename To, typename From>
+__device__ __forceinline__ To cvt(From v) { return To(v); }
+template <>
+__device__ __forceinline__ double cvt<double, float>(float v) {
+    double d;
+    asm("cvt.f64.f32 %0, %1;" : "=d"(d) : "f"(v));
+    return d;
+}
+template <>
+__device__ __forceinline__ float cvt<float, double>(double v) {
+    float f;
+    asm("cvt.rn.f32.f64 %0, %1;" : "=f"(f) : "d"(v));
+    return f;
+}
+
 // v[q] += sum_r Tm[q][r] * o[r]
 template <typename A, int K>
 __device__ __forceinline__ void matvec_acc(A (&v)[K], const A* Tm, const A (&o)[K]) {
@@ -701,14 +720,14 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             T t = tb.alpha[0] * xv[P + u];
 #pragma unroll
             for (int q = 1; q <= P; q++) t = mad(tb.alpha[q], xv[P + u - q], t);
-            A acc = A(t);
+            A acc = cvt<A, T>(t);
 #pragma unroll
             for (int r = K; r >= 1; r--)
                 if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
 #pragma unroll
             for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
             hist[0] = acc;
-            lf[u] = T(acc);
+            lf[u] = cvt<T, A>(acc);
         }
         A v[K];
 #pragma unroll
@@ -826,7 +845,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         }
         T Sd[K];
 #pragma unroll
-        for (int q = 0; q < K; q++) Sd[q] = T(Sst[q]);
+        for (int q = 0; q < K; q++) Sd[q] = cvt<T, A>(Sst[q]);
         T* base = st + kHalo + tid * X;
         T yv[X];
 #pragma unroll

@@ -350,7 +350,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         for (int r = 0; r < K; r++) hist[r] = A(0);
 #pragma unroll
         for (int u = 0; u < X; u++) {
-            A acc = A(fir(xv, u));
+            A acc = cvt<A, T>(fir(xv, u));
 #pragma unroll
             for (int r = K; r >= 1; r--)
                 if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
@@ -382,27 +382,46 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             for (int q = 0; q < K; q++) wagg[(slot * W + warp) * kMaxK + q] = v[q];
         }
         named_sync(1, NC);
-        // a4: scan of the W warp aggregates with T(32X * 2^s)
-        A u_[K];
+#ifndef PLR_RR_BLK1
+#define PLR_RR_BLK1 1
+#endif
+        // a4: scan of the W warp aggregates with T(32X * 2^s).  One warp per
+        // tile (rotating) scans and writes every warp's exclusive prefix; the
+        // other warps go straight on (their phase B reads sPw after the carry,
+        // ordered by agg_bar -> look-back -> carry_bar).  wagg[slot] / sPw[slot]
+        // are rewritten only after the named barrier of tile it+NS, which every
+        // warp reaches after its phase B of tile it.
+        if (!PLR_RR_BLK1 || warp == it % W) {
+            A u_[K];
 #pragma unroll
-        for (int q = 0; q < K; q++) u_[q] = lane < W ? wagg[(slot * W + lane) * kMaxK + q] : A(0);
+            for (int q = 0; q < K; q++) u_[q] = lane < W ? wagg[(slot * W + lane) * kMaxK + q] : A(0);
 #pragma unroll
-        for (int s2 = 0; s2 < LOGW; s2++) {
-            A o[K];
+            for (int s2 = 0; s2 < LOGW; s2++) {
+                A o[K];
 #pragma unroll
-            for (int q = 0; q < K; q++) o[q] = shfl_up(u_[q], 1 << s2);
-            if (lane >= (1 << s2)) matvec_acc<A, K>(u_, tb.Tblk[s2], o);
-        }
+                for (int q = 0; q < K; q++) o[q] = shfl_up(u_[q], 1 << s2);
+                if (lane >= (1 << s2)) matvec_acc<A, K>(u_, tb.Tblk[s2], o);
+            }
+            if (PLR_RR_BLK1) {
 #pragma unroll
-        for (int q = 0; q < K; q++) {
-            const A pw = shfl_idx(u_[q], (warp + 31) & 31);
-            const A at = shfl_idx(u_[q], W - 1);                // tile aggregate
-            if (lane == 0) sPw[(slot * W + warp) * K + q] = warp == 0 ? A(0) : pw;
-            if (tid == 0) sAt[slot * kMaxK + q] = at;
+                for (int q = 0; q < K; q++) {
+                    const A pw = shfl_up(u_[q], 1);
+                    if (lane < W) sPw[(slot * W + lane) * K + q] = lane == 0 ? A(0) : pw;
+                    if (lane == W - 1) sAt[slot * kMaxK + q] = u_[q];   // tile aggregate
+                }
+            } else {
+#pragma unroll
+                for (int q = 0; q < K; q++) {
+                    const A pw = shfl_idx(u_[q], (warp + 31) & 31);
+                    const A at = shfl_idx(u_[q], W - 1);            // tile aggregate
+                    if (lane == 0) sPw[(slot * W + warp) * K + q] = warp == 0 ? A(0) : pw;
+                    if (tid == 0) sAt[slot * kMaxK + q] = at;
+                }
+            }
         }
         tmem_wait_st();
         __syncwarp();
-        if (tid == 0) { slot_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
+        if (PLR_RR_BLK1 ? (warp == it % W && lane == 0) : tid == 0) { slot_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
         return j;
     };
 
@@ -439,13 +458,13 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         T yv[X];
 #pragma unroll
         for (int u = 0; u < X; u++) {
-            A acc = A(fir(xv, u));
+            A acc = cvt<A, T>(fir(xv, u));
 #pragma unroll
             for (int r = K; r >= 1; r--) acc = mad(tb.c[r - 1], S[r - 1], acc);
 #pragma unroll
             for (int r = K - 1; r >= 1; r--) S[r] = S[r - 1];
             S[0] = acc;
-            yv[u] = T(acc);
+            yv[u] = cvt<T, A>(acc);
         }
         // a7: y into the stage (TMA store by the storer) or global (ragged)
         if (!ragged) {

@@ -408,14 +408,14 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             T t = tb.alpha[0] * xv[P + u];
 #pragma unroll
             for (int q = 1; q <= P; q++) t = mad(tb.alpha[q], xv[P + u - q], t);
-            A acc = A(t);
+            A acc = cvt<A, T>(t);
 #pragma unroll
             for (int r = K; r >= 1; r--)
                 if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
 #pragma unroll
             for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
             hist[0] = acc;
-            w[u] = lo_word<T>(T(acc));
+            w[u] = lo_word<T>(cvt<T, A>(acc));
         }
         A v[K];
 #pragma unroll
@@ -491,7 +491,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         }
         T Sd[K];
 #pragma unroll
-        for (int q = 0; q < K; q++) Sd[q] = T(Sst[q]);
+        for (int q = 0; q < K; q++) Sd[q] = cvt<T, A>(Sst[q]);
         T yv[X];
 #pragma unroll
         for (int u = 0; u < X; u++) {
