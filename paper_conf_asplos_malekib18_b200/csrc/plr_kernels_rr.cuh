@@ -425,10 +425,13 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         return j;
     };
 
-    auto phaseB = [&](int it, long long j) {
+    auto phaseB = [&](int it) {
         const int slot = it % NS;
         const int sb = it % SB;
         mbar_wait(&carry_bar[slot], (uint32_t)((it / NS) & 1));
+        // the tile id is read after the carry wait: the block-scan warp of
+        // phase A wrote it before agg_bar, which the carry is ordered after
+        const long long j = slot_tile[slot];
         const bool ragged = (j == ntiles - 1) && last_ragged;
         const long long g0 = j * (long long)M + (long long)tid * X;
         uint32_t w[CW];
@@ -502,11 +505,11 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         if (phaseA(na) >= ntiles) break;
     for (bool stop = na < D; !stop;) {
         const long long j = phaseA(na);
-        phaseB(nb, slot_tile[nb % NS]);
+        phaseB(nb);
         nb++;
         if (j >= ntiles) stop = true; else na++;
     }
-    for (; nb < na; nb++) phaseB(nb, slot_tile[nb % NS]);      // drain
+    for (; nb < na; nb++) phaseB(nb);                           // drain
     // loader B, storer and look-back warps beyond the stop see *stop_pos
     tc_fence_before();
     named_sync(1, NC);

@@ -466,10 +466,13 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         return j;
     };
 
-    auto phaseB = [&](int it, long long j) {
+    auto phaseB = [&](int it) {
         const int slot = it % NT;
         const int sT = it % ST;
         mbar_wait(&carry_bar[slot], (uint32_t)((it / NT) & 1));
+        // tile id read after the carry wait (tid 0 wrote it before agg_bar,
+        // which the carry is ordered after; no barrier follows a stop)
+        const long long j = slot_tile[slot];
         const bool ragged = (j == ntiles - 1) && last_ragged;
         const long long g0 = j * (long long)M + (long long)tid * X;
         uint32_t w[CW];
@@ -536,11 +539,11 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         if (phaseA(na) >= ntiles) break;
     for (bool stop = na < D; !stop;) {
         const long long j = phaseA(na);
-        phaseB(nb, slot_tile[nb % NT]);
+        phaseB(nb);
         nb++;
         if (j >= ntiles) stop = true; else na++;
     }
-    for (; nb < na; nb++) phaseB(nb, slot_tile[nb % NT]);      // drain
+    for (; nb < na; nb++) phaseB(nb);                           // drain
     // stop markers: the storer, and look-back warps waiting beyond the stop
     {
         // no wait for the stage: only its id slot is written, and the storer
