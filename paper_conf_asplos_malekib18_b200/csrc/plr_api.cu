@@ -324,6 +324,11 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     // the DECAY specialisation (single-hop look-back) for this plan
     const char* fg = std::getenv("PLR_FORCE_GENERIC");
     const bool force_generic = fg != nullptr && fg[0] == '1';
+    if (st == PLR_OK && plan->pt.decay_flag && plan->pt.acc64 && !force_generic) {
+        // fp64-accumulation DECAY plans use their own tile geometry
+        plan_tables_free(&plan->pt);
+        st = plan_tables(a, p, b, k, dtype, class_geometry(true, k, true), &plan->pt, &why);
+    }
     if (st == PLR_OK && (!plan->pt.decay_flag || force_generic)) {
         plan_tables_free(&plan->pt);
         st = plan_tables(a, p, b, k, dtype, class_geometry(false, k), &plan->pt, &why);

@@ -3,9 +3,10 @@
 
 namespace plr {
 
-Geometry class_geometry(bool decay, int k) {
+Geometry class_geometry(bool decay, int k, bool acc64) {
     // x elements per thread (odd: conflict-free strided smem access) and W
     // compute warps per config; the ring depth is reported by scan_stages()
+    if (decay && acc64) return Geometry{inst::CfgDec64::X, inst::CfgDec64::W, inst::CfgDec64::S, 1};
     if (decay) return Geometry{inst::CfgDec::X, inst::CfgDec::W, inst::CfgDec::S, 1};
     switch (inst::gen_kind(k)) {
         case 2: return Geometry{PLR_RR_X, PLR_RR_W, PLR_RR_SA + PLR_RR_SB, PLR_RR_G};

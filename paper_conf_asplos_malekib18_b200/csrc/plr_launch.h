@@ -32,7 +32,8 @@ struct LaunchArgs {
 };
 
 // Tile geometry of the DECAY / generic kernel configs.
-Geometry class_geometry(bool decay, int k);
+// (fp64-accumulation DECAY plans have their own config)
+Geometry class_geometry(bool decay, int k, bool acc64 = false);
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm);

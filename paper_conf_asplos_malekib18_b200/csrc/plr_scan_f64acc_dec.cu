@@ -3,6 +3,6 @@
 
 namespace plr {
 cudaError_t launch_scan_f64acc_dec(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p) {
-    return inst::launch<float, double, inst::CfgDec>(tab, la, k, p);
+    return inst::launch<float, double, inst::CfgDec64>(tab, la, k, p);
 }
 }  // namespace plr

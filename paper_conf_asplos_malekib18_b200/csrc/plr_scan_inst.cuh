@@ -16,13 +16,24 @@ namespace inst {
 //     S = 4 stages, phase-A lead D = 1, one look-back warp;
 //   generic (multi-tile look-back): deep pipeline so predecessors' aggregates
 //     are published before a tile looks back: S = 6, D = 3, two look-back warps.
+//   fp32 DECAY: X = 23, W = 8 (tile 5888), 2 CTAs/SM; fp64-accumulation
+//   DECAY (issue-bound, R16): X = 31, W = 4 (tile 3968), 3 CTAs/SM, so the
+//   per-thread scan overhead is amortised over more elements (measured r01q).
 #ifndef PLR_DEC_S
 #define PLR_DEC_S 4
 #define PLR_DEC_D 1
 #define PLR_DEC_NL 1
-#define PLR_DEC_X 15
+#define PLR_DEC_X 23
 #define PLR_DEC_W 8
-#define PLR_DEC_MINB 3
+#define PLR_DEC_MINB 2
+#endif
+#ifndef PLR_DEC64_S
+#define PLR_DEC64_S 4
+#define PLR_DEC64_D 1
+#define PLR_DEC64_NL 1
+#define PLR_DEC64_X 31
+#define PLR_DEC64_W 4
+#define PLR_DEC64_MINB 3
 #endif
 #ifndef PLR_GEN_S
 #define PLR_GEN_S 3
@@ -81,6 +92,7 @@ struct Cfg {
     static constexpr bool DEC = DEC_;
 };
 using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true>;
+using CfgDec64 = Cfg<PLR_DEC64_S, PLR_DEC64_D, PLR_DEC64_NL, PLR_DEC64_X, PLR_DEC64_W, PLR_DEC64_MINB, true>;
 using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false>;
 
 template <typename T, typename A, int K>
