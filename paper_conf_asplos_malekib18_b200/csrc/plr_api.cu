@@ -66,6 +66,14 @@ static size_t elem_size(const plr_plan*) { return 4; }
 
 static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
+// Small-n launches use look-back units of one tile while the big-unit grid
+// would give each CTA fewer than one unit (tail imbalance);
+// PLR_UNIT1_WAVES overrides it (0: never) for size sweeps.
+static uint64_t unit1_waves() {
+    const char* e = std::getenv("PLR_UNIT1_WAVES");
+    return e != nullptr ? (uint64_t)std::strtoull(e, nullptr, 10) : (uint64_t)1;
+}
+
 // ============================================================ helpers =====
 namespace {
 
@@ -214,7 +222,12 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     if (n > plan->n_max) return fail(PLR_ERR_SIZE, "n exceeds the plan's n_max");
     const uint64_t m = (uint64_t)plan->pt.geo.tile();
     const uint64_t ntiles = (n + m - 1) / m;
-    const uint64_t G = (uint64_t)plan->pt.geo.G;            // tiles per ticket (look-back unit)
+    // tiles per ticket (look-back unit).  Small n: units of one tile, so the
+    // tiles spread over every SM (a unit of G tiles runs on one CTA);
+    // DECAY plans always have G = 1.
+    const uint64_t grid_max = (uint64_t)plan->num_sms * plan->ctas_per_sm;
+    const bool unit1 = plan->pt.geo.G > 1 && ntiles < unit1_waves() * grid_max * (uint64_t)plan->pt.geo.G;
+    const uint64_t G = unit1 ? 1 : (uint64_t)plan->pt.geo.G;
     const uint64_t nunits = (ntiles + G - 1) / G;
     if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
         CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, stream), "status reset");
@@ -224,7 +237,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         plan->dirty = false;
     }
     plan->epoch++;
-    const uint64_t grid = std::min<uint64_t>(nunits, (uint64_t)plan->num_sms * plan->ctas_per_sm);
+    const uint64_t grid = std::min<uint64_t>(nunits, grid_max);
     LaunchArgs la;
     la.x = x; la.y = y; la.n = n; la.ntiles = ntiles;
     la.ticket_base = plan->ticket_base;
@@ -240,6 +253,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.grid = (int)grid;
     la.sig = plan->sig_kernel ? plan->pt.sig_id : 0;
     la.store = store;
+    la.unit1 = unit1;
     la.stream = stream;
     cudaError_t e = launch_scan(plan->pt, la);
     if (e != cudaSuccess) {

@@ -24,9 +24,12 @@ int kernel_kind(const PlanTables& pt) {
 }
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la) {
-    if (pt.dtype == PLR_INT32) return launch_scan_i32(pt.ti, la, pt.k, pt.p);
-    if (pt.acc64) return pt.decay_flag ? launch_scan_f64acc_dec(pt.td, la, pt.k, pt.p)
-                                       : launch_scan_f64acc_gen(pt.td, la, pt.k, pt.p);
+    if (pt.dtype == PLR_INT32)
+        return la.unit1 ? launch_scan_i32_u1(pt.ti1, la, pt.k, pt.p) : launch_scan_i32(pt.ti, la, pt.k, pt.p);
+    if (pt.acc64) {
+        if (pt.decay_flag) return launch_scan_f64acc_dec(pt.td, la, pt.k, pt.p);
+        return la.unit1 ? launch_scan_f64acc_gen_u1(pt.td1, la, pt.k, pt.p) : launch_scan_f64acc_gen(pt.td, la, pt.k, pt.p);
+    }
     if (!pt.decay_flag) return cudaErrorInvalidValue;    // planner forces fp64 accumulation
     return launch_scan_f32(pt.tf, la, pt.k, pt.p);
 }

@@ -88,6 +88,8 @@ struct PlanTables {
     Tables<uint32_t, uint32_t> ti;       // int32 ring
     Tables<float, float> tf;             // fp32, fp32 accumulation
     Tables<float, double> td;            // fp32, fp64 accumulation
+    Tables<uint32_t, uint32_t> ti1;      // ti / td with look-back units of one tile (Tpow = T(m 2^s))
+    Tables<float, double> td1;
     uint32_t lane_i[kMaxK * kMaxK * 32];
     float lane_f[kMaxK * kMaxK * 32];
     double lane_d[kMaxK * kMaxK * 32];

@@ -27,6 +27,7 @@ struct LaunchArgs {
     int grid;
     int sig = 0;                        // compile-time signature id (plr_constsig.cuh), 0 = runtime tables
     bool store;
+    bool unit1 = false;                 // look-back units of one tile (small n): the *_u1 kernels
     cudaStream_t stream;
     int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel
 };
@@ -43,6 +44,8 @@ cudaError_t launch_scan_i32(const Tables<uint32_t, uint32_t>& tab, const LaunchA
 cudaError_t launch_scan_f32(const Tables<float, float>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t launch_scan_f64acc_dec(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t launch_scan_f64acc_gen(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_scan_i32_u1(const Tables<uint32_t, uint32_t>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_scan_f64acc_gen_u1(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
 // ring depth of the config a plan launches with (plan info)
 int scan_stages(const PlanTables& pt);
 // plr_plan_info.kernel_kind of a plan

@@ -195,6 +195,13 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         Mat<uint32_t> M = companion<uint32_t>(c, k);
         auto id = [](uint32_t v) { return v; };
         fill_tables(M, k, geo, &pt.ti, pt.lane_i, id, id);
+        {
+            Geometry g1 = geo;
+            g1.G = 1;
+            uint32_t lane_tmp[kMaxK * kMaxK * 32];
+            pt.ti1 = pt.ti;                    // coefficients (alpha, c); the matrices are refilled
+            fill_tables(M, k, g1, &pt.ti1, lane_tmp, id, id);
+        }
         // class: all factors 1 -> ONES; single unit feedback
         // coefficient -> PERM (0/1 repeating factors); otherwise POLY
         int nnz = 0, ones = 0;
@@ -228,6 +235,13 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         auto f64 = [](double v) { return std::fabs(v) < (double)FLT_MIN ? 0.0 : v; };
         fill_tables(M, k, geo, &pt.tf, pt.lane_f, f32, f32);
         fill_tables(M, k, geo, &pt.td, pt.lane_d, f32, f64);
+        {
+            Geometry g1 = geo;
+            g1.G = 1;
+            double lane_tmp[kMaxK * kMaxK * 32];
+            pt.td1 = pt.td;                    // coefficients (alpha, c); the matrices are refilled
+            fill_tables(M, k, g1, &pt.td1, lane_tmp, f32, f64);
+        }
         // DECAY: the fp32 impulse response g of (1: c) becomes
         // exactly 0 and stays 0.  g_0 = 1, g_u = sum_j c_j g_{u-j}.
         const int64_t cap = 1 << 16;

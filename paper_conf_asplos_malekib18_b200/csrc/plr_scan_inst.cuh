@@ -58,16 +58,19 @@ namespace inst {
 #define PLR_K1_KIND 1
 #endif
 #define PLR_GEN_TMEM (PLR_GEN_KIND != 0)
+// re-read kernel (measured r01r-r01u): X = 31, W = 8 (tile 7936), 3 look-back
+// warps, 2 HBM load stages, 5 L2 re-read / store stages, phase-B lag 8 tiles,
+// look-back units of 4 tiles (G >= 5 hung at NS = 9: not used)
 #ifndef PLR_RR_X
-#define PLR_RR_X 15
-#define PLR_RR_W 16
-#define PLR_RR_NL 2
-#define PLR_RR_SA 3         // phase-A (HBM) load stages
-#define PLR_RR_SB 4         // phase-B (L2 re-read + y store) stages
-#define PLR_RR_NS 7         // slots: phase B lags phase A by NS-1 tiles (L2 reuse distance)
+#define PLR_RR_X 31
+#define PLR_RR_W 8
+#define PLR_RR_NL 3
+#define PLR_RR_SA 2         // phase-A (HBM) load stages
+#define PLR_RR_SB 5         // phase-B (L2 re-read + y store) stages
+#define PLR_RR_NS 9         // slots: phase B lags phase A by NS-1 tiles (L2 reuse distance)
 #endif
 #ifndef PLR_RR_G
-#define PLR_RR_G 3          // tiles per look-back unit (one ticket, one look-back)
+#define PLR_RR_G 4          // tiles per look-back unit (one ticket, one look-back)
 #endif
 #ifndef PLR_TM_X
 #define PLR_TM_X 15
@@ -86,18 +89,22 @@ constexpr int gen_kind(int k) { return k == 1 ? PLR_K1_KIND : PLR_GEN_KIND; }
 // S-stage ring, phase-A lead D, NL look-back warps, X elements per thread,
 // W compute warps (tile m = 32 W X)
 // W compute warps (tile m = 32 W X); MINB: CTAs per SM the registers must allow
-template <int S_, int D_, int NL_, int X_, int W_, int MINB_, bool DEC_>
+// U1_: look-back units of one tile (the small-n launches, plr_api.cu), else
+// PLR_RR_G / PLR_TM_G tiles per unit
+template <int S_, int D_, int NL_, int X_, int W_, int MINB_, bool DEC_, bool U1_ = false>
 struct Cfg {
     static constexpr int S = S_, D = D_, NL = NL_, X = X_, W = W_, MINB = MINB_;
-    static constexpr bool DEC = DEC_;
+    static constexpr bool DEC = DEC_, U1 = U1_;
 };
 using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true>;
 using CfgDec64 = Cfg<PLR_DEC64_S, PLR_DEC64_D, PLR_DEC64_NL, PLR_DEC64_X, PLR_DEC64_W, PLR_DEC64_MINB, true>;
 using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false>;
+using CfgGen1 = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false, true>;
 
-template <typename T, typename A, int K>
+template <typename T, typename A, int K, bool U1>
 struct TmCfg {
-    static constexpr int X = PLR_TM_X, W = PLR_TM_W, NL = PLR_TM_NL, SL = PLR_TM_SL, ST = PLR_TM_ST, G = PLR_TM_G;
+    static constexpr int X = PLR_TM_X, W = PLR_TM_W, NL = PLR_TM_NL, SL = PLR_TM_SL, ST = PLR_TM_ST;
+    static constexpr int G = U1 ? 1 : PLR_TM_G;
     static constexpr int CW = dev::TmemCols<A, K, X>::CW;
 #ifndef PLR_TM_NTMAX
 #define PLR_TM_NTMAX 8
@@ -115,11 +122,11 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     void (*kern)(const ScanParams<T, A>);
     if constexpr (kind == 2) {
         kern = &dev::plr_scan_rr_kernel<T, A, K, P, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS, PLR_RR_NL,
-                                         PLR_RR_G, STORE, SIG>;
+                                         C::U1 ? 1 : PLR_RR_G, STORE, SIG>;
         smem = dev::LayoutR<T, A, K, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS>::bytes;
         threads = (PLR_RR_W + 1 + PLR_RR_NL) * 32;
     } else if constexpr (tmem) {
-        using TC = TmCfg<T, A, K>;
+        using TC = TmCfg<T, A, K, C::U1>;
         kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, TC::G, STORE, SIG>;
         smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
         threads = (TC::W + 1 + TC::NL) * 32;
