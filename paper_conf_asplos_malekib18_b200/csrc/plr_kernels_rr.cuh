@@ -87,6 +87,9 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                              : NS * WQ * CW <= 256 ? 256 : 512;   // power-of-two allocation
     static_assert(P <= kHalo, "halo");
     static_assert(G >= 1 && G <= kMaxG && G + 1 <= NS, "look-back unit of G tiles needs G+1 slots");
+    // guard: configurations with 2G > NS hung on B200 (r01u: re-read G = 5..8 at
+    // NS = 9; r01x: TMEM G = 4 at NT = 7); every shipped config satisfies it
+    static_assert(2 * G <= NS, "look-back unit too large for the slot ring");
     static_assert(SB >= 2 && SA >= 1, "stages");
     constexpr bool DEC = false;
 

@@ -170,6 +170,9 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     static_assert(NT >= 2 && NT * WQ * CW <= 512, "TMEM columns");
     static_assert(P <= kHalo, "halo");
     static_assert(G >= 1 && G <= kMaxG && G + 1 <= NT, "look-back unit of G tiles needs G+1 parked tiles");
+    // guard: configurations with 2G > NT hung on B200 (r01u: re-read G = 5..8 at
+    // NS = 9; r01x: TMEM G = 4 at NT = 7); every shipped config satisfies it
+    static_assert(2 * G <= NT, "look-back unit too large for the slot ring");
     constexpr bool DEC = false;
 
     extern __shared__ __align__(128) unsigned char smem[];
