@@ -612,10 +612,14 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 for (int q = 0; q < K; q++) Gp[q] = prm.y_hist != nullptr ? A(prm.y_hist[K - 1 - q]) : A(0);
             } else if (DEC) {
                 // T(m) == 0: every tile published inclusive == aggregate at
-                // once; the look-back is a single hop
+                // once; the look-back is a single hop.  Poll only
+                // once this tile's own phase A is done: its predecessor started
+                // at the same time, so it is (almost) always published by then
+                // and the poll does not steal issue slots from the compute warps.
+                mbar_wait(&agg_bar[slot], (uint32_t)((it / NS) & 1));
                 A v[K];
                 if (lane == 0) {
-                    int ns = 16;
+                    int ns = 64;
                     while (read_status<A, K, DEC>(prm.status, prm.status_mask, j - 1, v, tagA, tagI) != 2) {
                         __nanosleep(ns);
                         ns = ns < 256 ? 2 * ns : ns;
