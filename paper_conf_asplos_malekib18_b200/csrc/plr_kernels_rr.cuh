@@ -122,34 +122,6 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     constexpr Tables<T, A> kTab = const_tables<T, A>(SIG, X, W, G);
     static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
     const Tables<T, A>& tb = SIG != 0 ? kTab : prm.tab;
-    // binomial POLY rows of Table 1 evaluated as cascaded running sums
-    // (exact in Z/2^32, the same residues as the companion form)
-    constexpr bool kCascade = (SIG == kSigOrder2 && K == 2) || (SIG == kSigOrder3 && K == 3);
-    // cascade sums (c1 = K-th difference level ... c_K = y) <-> companion
-    // state (y_{u}, y_{u-1}, y_{u-2}): c_K = y_u, c_{K-1} = y_u - y_{u-1},
-    // c_{K-2} = y_u - 2 y_{u-1} + y_{u-2}
-    auto cascade_to_state = [](A c1, A c2, A c3, A (&v)[K]) {
-        if constexpr (K == 2) {
-            v[0] = c2;
-            v[1] = c2 - c1;
-        } else if constexpr (K == 3) {
-            v[0] = c3;
-            v[1] = c3 - c2;
-            v[2] = c3 - c2 - c2 + c1;
-        }
-        (void)c3;
-    };
-    auto state_to_cascade = [](const A (&v)[K], A& c1, A& c2, A& c3) {
-        if constexpr (K == 2) {
-            c2 = v[0];
-            c1 = v[0] - v[1];
-            c3 = A(0);
-        } else if constexpr (K == 3) {
-            c3 = v[0];
-            c2 = v[0] - v[1];
-            c1 = v[0] - v[1] - v[1] + v[2];
-        }
-    };
 
     if (tid == 0) {
         for (int s = 0; s < SA; s++) { mbar_init(&fullA[s], 1); mbar_init(&emptyA[s], NC); }
@@ -376,36 +348,22 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         read_x(stA + (size_t)s * SWL, j, ragged, xv);
         mbar_arrive(&emptyA[s]);                                // the stage may be refilled
         // a2: chunk end state with zero state (only the last K values matter)
-        A v[K];
-        if constexpr (kCascade) {
-            // (1: 2, -1) / (1: 3, -3, 1) = K-fold prefix sum: K
-            // cascaded running sums, one add each per element (no multiply,
-            // one add of latency per element on the serial path)
-            A c1 = A(0), c2 = A(0), c3 = A(0);
+        A hist[K];
 #pragma unroll
-            for (int u = 0; u < X; u++) {
-                c1 += cvt<A, T>(fir(xv, u));
-                c2 += c1;
-                if constexpr (K == 3) c3 += c2;
-            }
-            cascade_to_state(c1, c2, c3, v);
-        } else {
-            A hist[K];
+        for (int r = 0; r < K; r++) hist[r] = A(0);
 #pragma unroll
-            for (int r = 0; r < K; r++) hist[r] = A(0);
+        for (int u = 0; u < X; u++) {
+            A acc = cvt<A, T>(fir(xv, u));
 #pragma unroll
-            for (int u = 0; u < X; u++) {
-                A acc = cvt<A, T>(fir(xv, u));
+            for (int r = K; r >= 1; r--)
+                if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
 #pragma unroll
-                for (int r = K; r >= 1; r--)
-                    if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
-#pragma unroll
-                for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
-                hist[0] = acc;
-            }
-#pragma unroll
-            for (int q = 0; q < K; q++) v[q] = hist[q];
+            for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
+            hist[0] = acc;
         }
+        A v[K];
+#pragma unroll
+        for (int q = 0; q < K; q++) v[q] = hist[q];
         // a3: warp inclusive scan with T(X * 2^s)
 #pragma unroll
         for (int s2 = 0; s2 < 5; s2++) {
@@ -504,29 +462,15 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         read_x(st, j, ragged, xv);
         if constexpr (P > 0) named_sync(2, NC);                 // halo reads before y overwrites x
         T yv[X];
-        if constexpr (kCascade) {
-            // seed the cascaded sums with the backward differences of the
-            // incoming state (y_{-1}, y_{-2}, y_{-3})
-            A c1, c2, c3;
-            state_to_cascade(S, c1, c2, c3);
 #pragma unroll
-            for (int u = 0; u < X; u++) {
-                c1 += cvt<A, T>(fir(xv, u));
-                c2 += c1;
-                if constexpr (K == 3) c3 += c2;
-                yv[u] = cvt<T, A>(K == 3 ? c3 : c2);
-            }
-        } else {
+        for (int u = 0; u < X; u++) {
+            A acc = cvt<A, T>(fir(xv, u));
 #pragma unroll
-            for (int u = 0; u < X; u++) {
-                A acc = cvt<A, T>(fir(xv, u));
+            for (int r = K; r >= 1; r--) acc = mad(tb.c[r - 1], S[r - 1], acc);
 #pragma unroll
-                for (int r = K; r >= 1; r--) acc = mad(tb.c[r - 1], S[r - 1], acc);
-#pragma unroll
-                for (int r = K - 1; r >= 1; r--) S[r] = S[r - 1];
-                S[0] = acc;
-                yv[u] = cvt<T, A>(acc);
-            }
+            for (int r = K - 1; r >= 1; r--) S[r] = S[r - 1];
+            S[0] = acc;
+            yv[u] = cvt<T, A>(acc);
         }
         // a7: y into the stage (TMA store by the storer) or global (ragged)
         if (!ragged) {
