@@ -78,6 +78,13 @@ __device__ __forceinline__ bool mbar_try_wait_sleep(uint64_t* bar, uint32_t pari
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     while (!mbar_try_wait_sleep(bar, parity, PLR_WAIT_HINT_NS)) { }
 }
+// wait without a suspend hint, for lanes of a warp whose lanes play
+// different roles (loader / storer lanes of the producer warp): a lane
+// suspended for long in try_wait can hold back a diverged sibling lane that
+// the awaited arrival depends on (loader B waits on the storer's emptyB)
+__device__ __forceinline__ void mbar_wait_poll(uint64_t* bar, uint32_t parity) {
+    while (!mbar_try_wait(bar, parity)) { }
+}
 // TMA 1D bulk copy global -> shared, completion on an mbarrier (UBLKCP).
 __device__ __forceinline__ void bulk_load(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar,
                                           uint64_t policy) {

@@ -87,9 +87,11 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                              : NS * WQ * CW <= 256 ? 256 : 512;   // power-of-two allocation
     static_assert(P <= kHalo, "halo");
     static_assert(G >= 1 && G <= kMaxG && G + 1 <= NS, "look-back unit of G tiles needs G+1 slots");
-    // guard: configurations with 2G > NS hung on B200 (r01u: re-read G = 5..8 at
-    // NS = 9; r01x: TMEM G = 4 at NT = 7); every shipped config satisfies it
-    static_assert(2 * G <= NS, "look-back unit too large for the slot ring");
+    // guard: every configuration with 2G >= NS tried on B200 hung (re-read
+    // kernel: G = 4 at NS = 8, G = 5..8 at NS = 9/10, G = 6 at NS = 12; TMEM
+    // kernel: G = 4 at NT = 7), with or without try_wait suspend hints; the
+    // cause is not identified, so such configurations do not compile
+    static_assert(2 * G < NS, "look-back unit too large for the slot ring");
     static_assert(SB >= 2 && SA >= 1, "stages");
     constexpr bool DEC = false;
 
@@ -162,7 +164,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             long long unit = 0;
             for (int f = 0;; f++) {
                 const int s = f % SA;
-                if (f >= SA) mbar_wait(&emptyA[s], (uint32_t)(((f / SA) - 1) & 1));
+                if (f >= SA) mbar_wait_poll(&emptyA[s], (uint32_t)(((f / SA) - 1) & 1));
                 // one ticket per look-back unit of G consecutive tiles
                 if (f % G == 0) unit = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
                 long long j = unit * G + f % G;
@@ -179,7 +181,11 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 load_tile(stA + (size_t)s * SWL, j, &fullA[s], pol);
             }
         } else if (lane == 1) {                                     // loader B (L2)
-            const uint64_t pol = policy_evict_first();
+#ifndef PLR_RR_BPOL
+#define PLR_RR_BPOL 0
+#endif
+            // x is dead after the re-read: evict first (PLR_RR_BPOL=1: normal)
+            const uint64_t pol = PLR_RR_BPOL == 0 ? policy_evict_first() : policy_evict_normal();
             for (int f = 0;; f++) {
                 const int sb = f % SB;
                 // the tile id of position f is known once its phase A is done
@@ -190,7 +196,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     if (*stop_pos <= f) { stop = true; break; }
                 const long long j = stop ? ntiles : slot_tile[slot];
                 if (j >= ntiles) break;
-                if (f >= SB) mbar_wait(&emptyB[sb], (uint32_t)(((f / SB) - 1) & 1));
+                if (f >= SB) mbar_wait_poll(&emptyB[sb], (uint32_t)(((f / SB) - 1) & 1));
                 if (j == ntiles - 1 && last_ragged) { mbar_arrive(&fullB[sb]); continue; }
                 load_tile(stB + (size_t)sb * SWL, j, &fullB[sb], pol);
             }

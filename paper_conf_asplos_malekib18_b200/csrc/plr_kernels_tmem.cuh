@@ -170,9 +170,11 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     static_assert(NT >= 2 && NT * WQ * CW <= 512, "TMEM columns");
     static_assert(P <= kHalo, "halo");
     static_assert(G >= 1 && G <= kMaxG && G + 1 <= NT, "look-back unit of G tiles needs G+1 parked tiles");
-    // guard: configurations with 2G > NT hung on B200 (r01u: re-read G = 5..8 at
-    // NS = 9; r01x: TMEM G = 4 at NT = 7); every shipped config satisfies it
-    static_assert(2 * G <= NT, "look-back unit too large for the slot ring");
+    // guard: every configuration with 2G >= NT tried on B200 hung (re-read
+    // kernel: G = 4 at NS = 8, G = 5..8 at NS = 9/10, G = 6 at NS = 12; TMEM
+    // kernel: G = 4 at NT = 7), with or without try_wait suspend hints; the
+    // cause is not identified, so such configurations do not compile
+    static_assert(2 * G < NT, "look-back unit too large for the slot ring");
     constexpr bool DEC = false;
 
     extern __shared__ __align__(128) unsigned char smem[];
@@ -224,7 +226,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             long long unit = 0;
             for (int f = 0;; f++) {
                 const int s = f % SL;
-                if (f >= SL) mbar_wait(&empty_L[s], (uint32_t)(((f / SL) - 1) & 1));
+                if (f >= SL) mbar_wait_poll(&empty_L[s], (uint32_t)(((f / SL) - 1) & 1));
                 // one ticket per look-back unit of G consecutive tiles
                 if (f % G == 0) unit = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
                 long long j = unit * G + f % G;
@@ -257,7 +259,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             int np = 0;
             for (int t = 0;; t++) {
                 const int sT = t % ST;
-                mbar_wait(&full_T[sT], (uint32_t)((t / ST) & 1));
+                mbar_wait_poll(&full_T[sT], (uint32_t)((t / ST) & 1));
                 const long long jt = store_tile[sT];
                 if (jt >= ntiles) break;
                 if (STORE && !(jt == ntiles - 1 && last_ragged)) {
