@@ -138,6 +138,11 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     tc_fence_after();
     const uint32_t tmem_base = *tmem_base_p;
 
+    // phase B is needed for every tile when y is stored, else only for the
+    // tiles that hold y_{n-K} .. y_{n-1} (the end state the reduce returns)
+    auto covers_tail = [&](long long jj) -> bool {
+        return STORE || n < (unsigned long long)K || (unsigned long long)(jj + 1) * M > n - K;
+    };
     // TMA load of tile j (with its P-word halo) into stage st, completion on bar
     auto load_tile = [&](T* st, long long j, uint64_t* bar, uint64_t pol) {
         if (j == 0) {
@@ -198,6 +203,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 if (j >= ntiles) break;
                 if (f >= SB) mbar_wait_poll(&emptyB[sb], (uint32_t)(((f / SB) - 1) & 1));
                 if (j == ntiles - 1 && last_ragged) { mbar_arrive(&fullB[sb]); continue; }
+                if (!covers_tail(j)) { mbar_arrive(&fullB[sb]); continue; }   // reduce-only: phase B skipped
                 load_tile(stB + (size_t)sb * SWL, j, &fullB[sb], pol);
             }
         } else if (lane == 2) {                                     // storer
@@ -441,6 +447,15 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         // the tile id is read after the carry wait: the block-scan warp of
         // phase A wrote it before agg_bar, which the carry is ordered after
         const long long j = slot_tile[slot];
+        if (!covers_tail(j)) {
+            // reduce-only launch (STORE = false, the sharded schedule's first
+            // pass): only the tiles holding the last K outputs (y_tail) need
+            // phase B; the others keep the stage protocol and do no work
+            mbar_wait(&fullB[sb], (uint32_t)((it / SB) & 1));
+            if (tid == 0) store_tile[sb] = j;
+            mbar_arrive(&yfull[sb]);
+            return;
+        }
         const bool ragged = (j == ntiles - 1) && last_ragged;
         const long long g0 = j * (long long)M + (long long)tid * X;
         uint32_t w[CW];
