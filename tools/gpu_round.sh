@@ -15,6 +15,9 @@ if [ -z "$NONCU" ]; then
   bash tools/ncu_profile.sh ${TAG} "${NCU_SIGS:-tuple2 tuple3}"
 fi
 if [ -z "$NOEXTRA" ]; then
+  timeout 300 python tools/small_n.py > gpurun_out/${TAG}_small_n_host.jsonl 2>&1
+  SMALLN_HOST=0 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_small_n.csv python tools/small_n.py > gpurun_out/${TAG}_small_n_ncu.log 2>&1
+  python tools/small_n.py --parse gpurun_out/${TAG}_small_n.csv > gpurun_out/${TAG}_small_n.md 2>&1
   timeout 600 python tools/ablation.py > gpurun_out/${TAG}_ablation.jsonl 2> gpurun_out/${TAG}_ablation.err
   timeout 600 python tools/sweep.py > gpurun_out/${TAG}_sweep.jsonl 2> gpurun_out/${TAG}_sweep.err
 fi
