@@ -104,6 +104,40 @@ def test_repeated_launches_epochs(cuda_plr, sig):
 
 
 @pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+@pytest.mark.parametrize("n", [5000, 3 * M + 7, (1 << 20) + 12345])
+def test_cuda_graph_replay(cuda_plr, sig, n):
+    """plr_execute captured in a CUDA graph: the ticket base and the epoch
+    live on the device (launch_state_advance), so every replay, and eager
+    launches of the same plan between replays, see a fresh launch state."""
+    import torch
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    xd = torch.from_numpy(workloads.host_input(n, sig.dtype, 300)).cuda()
+    yd = torch.empty_like(xd)
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        plan(xd, yd)                                     # warm-up outside the capture
+    torch.cuda.current_stream().wait_stream(s)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        plan(xd, yd)
+    for t in range(4):
+        x = workloads.host_input(n, sig.dtype, 301 + t)
+        xd.copy_(torch.from_numpy(x))
+        for _ in range(t + 1):                           # repeated replays of the same launch
+            g.replay()
+        check(yd.cpu().numpy(), oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype,
+              "%s graph replay %d n=%d" % (sig.name, t, n))
+        m = max(1, n // (t + 2))                         # an eager launch of another size in between
+        ye = plan(xd[:m]).cpu().numpy()
+        check(ye, oracle.recurrence(x[:m], sig.a, sig.b, sig.dtype), sig.dtype,
+              "%s eager after replay %d m=%d" % (sig.name, t, m))
+    del g
+    plan.close()
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
 def test_continue_chunks(cuda_plr, sig):
     """plr_execute_continue over chunks (history = preceding inputs/outputs)
     equals one call (P:78 zero state only at the very start)."""

@@ -89,8 +89,22 @@ def run():
                     plan(x, y)
                 e1.record()
                 torch.cuda.synchronize()
-                print(json.dumps({"sig": name, "n": n, "back_to_back_us_per_call": round(e0.elapsed_time(e1) * 5, 2)}),
-                      flush=True)
+                b2b = e0.elapsed_time(e1) * 5
+                # the same launch captured 20x in a CUDA graph (launch state lives on the device)
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g):
+                    for _ in range(20):
+                        plan(x, y)
+                g.replay()
+                torch.cuda.synchronize()
+                e0.record()
+                for _ in range(10):
+                    g.replay()
+                e1.record()
+                torch.cuda.synchronize()
+                print(json.dumps({"sig": name, "n": n, "back_to_back_us_per_call": round(b2b, 2),
+                                  "graph_us_per_call": round(e0.elapsed_time(e1) * 1000 / 200, 2)}), flush=True)
+                del g
     for p in plans.values():
         p.close()
 
