@@ -34,6 +34,11 @@
  *  - A plan is like a cuFFT plan: it owns its scratch (tile-status words,
  *    ticket counter, tables, payload buffers) and must be used on one
  *    stream at a time.
+ *  - plr_execute, plr_execute_continue and plr_reduce may be captured in a
+ *    CUDA graph (stream capture) after one eager call on the plan: the
+ *    per-launch state (ticket base, status epoch) lives in device memory and
+ *    each launch advances it for the next, so replays and eager launches of
+ *    the same plan can be interleaved in stream order.
  */
 #ifndef PLR_H
 #define PLR_H

@@ -41,9 +41,8 @@ struct plr_plan {
     uint64_t max_tiles = 0;
     uint64_t status_slots = 0;              // power of two >= max_tiles
     unsigned long long* d_ticket = nullptr;
-    unsigned long long ticket_base = 0;
     unsigned long long* d_status = nullptr;
-    uint32_t epoch = 0;
+    uint32_t epoch = 0;                 // host count of launches since the last reset (overflow guard)
     void* d_lane = nullptr;
     float* d_fix = nullptr;
     bool dirty = false;
@@ -63,6 +62,10 @@ struct plr_plan {
 };
 
 static size_t elem_size(const plr_plan*) { return 4; }
+
+// ticket counter, launch base, epoch: the launch state lives on the device
+// (launch_state_advance), so plr_execute can be captured in a CUDA graph
+static constexpr size_t kTicketBytes = 3 * sizeof(unsigned long long);
 
 static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
@@ -231,20 +234,17 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     const uint64_t nunits = (ntiles + G - 1) / G;
     if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
         CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, stream), "status reset");
-        CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, 8, stream), "ticket reset");
+        CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, kTicketBytes, stream), "ticket reset");
         plan->epoch = 0;
-        plan->ticket_base = 0;
         plan->dirty = false;
     }
     plan->epoch++;
     const uint64_t grid = std::min<uint64_t>(nunits, grid_max);
     LaunchArgs la;
     la.x = x; la.y = y; la.n = n; la.ntiles = ntiles;
-    la.ticket_base = plan->ticket_base;
     la.ticket = plan->d_ticket;
     la.status = plan->d_status;
     la.status_mask = plan->status_slots - 1;
-    la.epoch = plan->epoch;
     la.decay = plan->pt.decay_flag;
     la.dec_mask = plan->pt.dec_mask;
     la.x_hist = x_hist; la.y_hist = y_hist; la.y_tail = y_tail;
@@ -260,7 +260,6 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         plan->dirty = true;
         return cuda_fail(e, "scan kernel launch");
     }
-    plan->ticket_base += nunits + grid;   // each CTA makes exactly one failing grab
     return PLR_OK;
 }
 
@@ -383,9 +382,9 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     if (plan->max_tiles > (1ull << 31)) { plr_plan_destroy(plan); return fail(PLR_ERR_SIZE, "n_max too large"); }
     plan->status_slots = 1;
     while (plan->status_slots < plan->max_tiles) plan->status_slots <<= 1;
-    if ((e = cudaMalloc(&plan->d_ticket, 8)) != cudaSuccess) return bail(e, "alloc ticket");
+    if ((e = cudaMalloc(&plan->d_ticket, kTicketBytes)) != cudaSuccess) return bail(e, "alloc ticket");
     if ((e = cudaMalloc(&plan->d_status, plan->status_slots * kStatusMaxBytes)) != cudaSuccess) return bail(e, "alloc status");
-    if ((e = cudaMemset(plan->d_ticket, 0, 8)) != cudaSuccess) return bail(e, "memset");
+    if ((e = cudaMemset(plan->d_ticket, 0, kTicketBytes)) != cudaSuccess) return bail(e, "memset");
     if ((e = cudaMemset(plan->d_status, 0, plan->status_slots * kStatusMaxBytes)) != cudaSuccess) return bail(e, "memset");
     const bool acc64 = dtype == PLR_FLOAT32 && plan->pt.acc64;
     const size_t lane_bytes = (size_t)k * k * 32 * (acc64 ? 8 : 4);

@@ -56,11 +56,9 @@ struct ScanParams {
     T* y;
     uint64_t n;
     uint64_t ntiles;
-    unsigned long long ticket_base;
-    unsigned long long* ticket;
+    unsigned long long* ticket;          // [0] counter, [1] launch base, [2] epoch (launch_state_advance)
     unsigned long long* status;          // 2^c scattered records of {tag:32 | value:32} words
     uint32_t status_mask;                // 2^c - 1, 2^c >= ntiles
-    uint32_t epoch;                      // tags 2*epoch (aggregate) / 2*epoch+1 (inclusive)
     int decay;                           // T(m) == 0 exactly: inclusive == aggregate
     uint32_t dec_mask;                   // DECAY kernels: bit s < 5 = lane-scan step s has a non-negligible
                                          // T(X 2^s); bit 5 = warp-aggregate level (T(32X d), d >= 1) non-negligible

@@ -31,6 +31,24 @@
 namespace plr {
 namespace dev {
 
+// ------------------------------------------------------ launch state -------
+// ticket[0] = ticket counter, ticket[1] = this launch's ticket base,
+// ticket[2] = the previous launch's epoch.  Every CTA makes exactly one
+// failing grab, so a launch takes total = units + grid tickets; the grab with
+// relative index total - 1 is the last one and advances the state for the
+// next launch on the stream.  Nothing of a launch lives on the host, so a
+// launch captured in a CUDA graph replays correctly.
+__device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long* p) {
+    return *reinterpret_cast<const volatile unsigned long long*>(p);
+}
+__device__ __forceinline__ void launch_state_advance(unsigned long long* tk, long long rel, unsigned long long total,
+                                                     unsigned long long base, uint32_t epoch) {
+    if ((unsigned long long)rel == total - 1) {
+        reinterpret_cast<volatile unsigned long long*>(tk)[1] = base + total;
+        reinterpret_cast<volatile unsigned long long*>(tk)[2] = epoch;
+    }
+}
+
 // ---------------------------------------------------------------- PTX ------
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
@@ -538,6 +556,12 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const bool last_ragged = (n % (unsigned long long)M) != 0;
     const Tables<T, A>& tb = prm.tab;
 
+    // launch state from device memory (tickets, epoch); the barrier consumes
+    // the loads, so they complete before this CTA's first ticket grab
+    const unsigned long long tbase = ld_volatile_u64(prm.ticket + 1);
+    const uint32_t epoch = (uint32_t)ld_volatile_u64(prm.ticket + 2) + 1u;
+    (void)__syncthreads_or((int)(tbase == 0ull && epoch == 0u));
+
     if (tid == 0) {
         for (int s = 0; s < S; s++) { mbar_init(&full_bar[s], 1); mbar_init(&done_bar[s], NC); }
         for (int s = 0; s < NS; s++) { mbar_init(&agg_bar[s], 1); mbar_init(&carry_bar[s], 1); }
@@ -559,9 +583,12 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 mbar_arrive(&full_bar[s]);
                 return;
             }
-            const long long j = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
+            const long long j = (long long)(atomicAdd(prm.ticket, 1ull) - tbase);
             tile_of[s] = j;
-            if (j >= ntiles) { stop_at = idx; mbar_arrive(&full_bar[s]); return; }
+            if (j >= ntiles) {
+                launch_state_advance(prm.ticket, j, (unsigned long long)ntiles + gridDim.x, tbase, epoch);
+                stop_at = idx; mbar_arrive(&full_bar[s]); return;
+            }
             if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_bar[s]); return; }   // compute loads it
             T* st = stages + (size_t)s * SW;
             if (j == 0) {
@@ -603,7 +630,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // the full barrier (as soon as the tile is loaded) and walks back without
     // waiting for the tile's own aggregate, which the compute warps publish.
     if (warp > W) {
-        const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
+        const uint32_t tagA = 2u * epoch, tagI = 2u * epoch + 1u;
         static_assert(NL <= kMaxNL, "look-back warps");
         const LbStats lbs{reinterpret_cast<unsigned long long*>(smem + L::off_lbstat) + (warp - W - 1) * kLbStatWords};
         lbs.init(lane);
@@ -786,7 +813,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 A At[K];
 #pragma unroll
                 for (int q = 0; q < K; q++) At[q] = wagg[(slot * W + W - 1) * kMaxK + q];
-                publish_status<A, K, DEC>(prm.status, prm.status_mask, j, At, 2u * prm.epoch + 1u, lane);
+                publish_status<A, K, DEC>(prm.status, prm.status_mask, j, At, 2u * epoch + 1u, lane);
             }
             __syncwarp();
             if (tid == 0) { agg_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
@@ -816,7 +843,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             A At[K];
 #pragma unroll
             for (int q = 0; q < K; q++) At[q] = shfl_idx(u_[q], W - 1);
-            publish_status<A, K, DEC>(prm.status, prm.status_mask, j, At, DEC ? 2u * prm.epoch + 1u : 2u * prm.epoch, lane);
+            publish_status<A, K, DEC>(prm.status, prm.status_mask, j, At, DEC ? 2u * epoch + 1u : 2u * epoch, lane);
         }
         // wagg is buffered per slot: its next writer (tile it+NS) runs after
         // every warp passed tile it+1's barrier

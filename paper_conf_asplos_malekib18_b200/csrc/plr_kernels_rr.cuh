@@ -125,6 +125,12 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
     const Tables<T, A>& tb = SIG != 0 ? kTab : prm.tab;
 
+    // launch state from device memory (tickets, epoch); the barrier consumes
+    // the loads, so they complete before this CTA's first ticket grab
+    const unsigned long long tbase = ld_volatile_u64(prm.ticket + 1);
+    const uint32_t epoch = (uint32_t)ld_volatile_u64(prm.ticket + 2) + 1u;
+    (void)__syncthreads_or((int)(tbase == 0ull && epoch == 0u));
+
     if (tid == 0) {
         for (int s = 0; s < SA; s++) { mbar_init(&fullA[s], 1); mbar_init(&emptyA[s], NC); }
         for (int s = 0; s < SB; s++) { mbar_init(&fullB[s], 1); mbar_init(&emptyB[s], 1); mbar_init(&yfull[s], NC); }
@@ -171,14 +177,16 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 const int s = f % SA;
                 if (f >= SA) mbar_wait_poll(&emptyA[s], (uint32_t)(((f / SA) - 1) & 1));
                 // one ticket per look-back unit of G consecutive tiles
-                if (f % G == 0) unit = (long long)(atomicAdd(prm.ticket, 1ull) - prm.ticket_base);
+                if (f % G == 0) unit = (long long)(atomicAdd(prm.ticket, 1ull) - tbase);
                 long long j = unit * G + f % G;
                 if (j >= ntiles) j = ntiles;
                 tileA[s] = j;
                 if (j >= ntiles) {
                     // the CTA that ends inside the last (partial) unit still makes
                     // its one failing grab: the host counts nunits + grid tickets
-                    if (f % G != 0) atomicAdd(prm.ticket, 1ull);
+                    const long long rel = f % G != 0 ? (long long)(atomicAdd(prm.ticket, 1ull) - tbase) : unit;
+                    launch_state_advance(prm.ticket, rel, (unsigned long long)((ntiles + G - 1) / G) + gridDim.x,
+                                         tbase, epoch);
                     mbar_arrive(&fullA[s]);
                     break;
                 }
@@ -240,7 +248,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // every tile its carry-in L_{g-1} + T(g m) G_{J-1} and publish the unit's
     // inclusive carry L_{G-1} + T(G m) G_{J-1}.
     if (warp > W) {
-        const uint32_t tagA = 2u * prm.epoch, tagI = 2u * prm.epoch + 1u;
+        const uint32_t tagA = 2u * epoch, tagI = 2u * epoch + 1u;
         static_assert(NL <= kMaxNL, "look-back warps");
         const LbStats lbs{reinterpret_cast<unsigned long long*>(smem + L::off_lbstat) + (warp - W - 1) * kLbStatWords};
         lbs.init(lane);

@@ -12,11 +12,9 @@ struct LaunchArgs {
     void* y;
     uint64_t n;
     uint64_t ntiles;
-    unsigned long long ticket_base;
     unsigned long long* ticket;
     unsigned long long* status;
     uint32_t status_mask;
-    uint32_t epoch;
     int decay;
     uint32_t dec_mask = 0x3f;
     const void* x_hist;

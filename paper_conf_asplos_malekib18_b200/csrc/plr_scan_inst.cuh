@@ -151,11 +151,9 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     prm.y = static_cast<T*>(la.y);
     prm.n = la.n;
     prm.ntiles = la.ntiles;
-    prm.ticket_base = la.ticket_base;
     prm.ticket = la.ticket;
     prm.status = la.status;
     prm.status_mask = la.status_mask;
-    prm.epoch = la.epoch;
     prm.decay = la.decay;
     prm.dec_mask = la.dec_mask;
     prm.x_hist = static_cast<const T*>(la.x_hist);
