@@ -161,7 +161,7 @@ class Plan:
         _check(lib.plr_plan_debug_stats(self._h, buf, int(reset)), "plr_plan_debug_stats")
         return {"lookbacks": buf[0], "windows": buf[1], "waits": buf[2], "depth_sum": buf[3],
                 "cyc_agg": buf[4], "cyc_lookback": buf[5], "cyc_sleep": buf[6], "cyc_load": buf[7],
-                "cyc_fold": buf[8]}
+                "cyc_fold": buf[8], "trace": [buf[i] for i in range(9, 16)]}
 
     def factor_lists(self, m: int):
         """The k seed-extended correction-factor lists (Sec. 2.1) as planned."""

@@ -437,7 +437,7 @@ plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out, int reset) {
         memset(out, 0, 16 * sizeof(uint64_t));
         return PLR_OK;
     }
-    CUDA_TRY(cudaMemcpy(out, plan->d_stats, 64, cudaMemcpyDeviceToHost), "stats copy");
+    CUDA_TRY(cudaMemcpy(out, plan->d_stats, 128, cudaMemcpyDeviceToHost), "stats copy");
     if (reset) CUDA_TRY(cudaMemset(plan->d_stats, 0, 128), "stats reset");
     return PLR_OK;
 }

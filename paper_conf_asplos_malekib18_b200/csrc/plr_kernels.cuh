@@ -49,6 +49,15 @@ __device__ __forceinline__ void launch_state_advance(unsigned long long* tk, lon
     }
 }
 
+// PLR_TRACE builds (experiment variants only): globaltimer stamps of CTA 0's
+// single-tile critical path into stats words 9..15 (plan made with PLR_STATS=1)
+#ifdef PLR_TRACE
+#define PLR_STAMP(i) do { if (prm.stats != nullptr && blockIdx.x == 0) { unsigned long long t_; \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_)); prm.stats[i] = t_; } } while (0)
+#else
+#define PLR_STAMP(i) do { } while (0)
+#endif
+
 // ---------------------------------------------------------------- PTX ------
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);

@@ -125,6 +125,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
     const Tables<T, A>& tb = SIG != 0 ? kTab : prm.tab;
 
+    if (threadIdx.x == 0) PLR_STAMP(10);
     // launch state from device memory (tickets, epoch); the barrier consumes
     // the loads, so they complete before this CTA's first ticket grab
     const unsigned long long tbase = ld_volatile_u64(prm.ticket + 1);
@@ -143,6 +144,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_base_p;
+    if (tid == 0) PLR_STAMP(9);
 
     // phase B is needed for every tile when y is stored, else only for the
     // tiles that hold y_{n-K} .. y_{n-1} (the end state the reduce returns)
@@ -236,6 +238,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 mbar_arrive(&emptyB[sb]);
             }
             bulk_wait_all<0>();
+            PLR_STAMP(14);
         }
         return;
     }
@@ -315,6 +318,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             matvec_acc<A, K>(Gi, tb.Tpow[0], Gp);              // G_J = L_{G-1} + T(G m) G_{J-1}
             publish_status<A, K, DEC>(prm.status, prm.status_mask, J, Gi, tagI, lane);
         }
+        if (warp == W + 1 && lane == 0) PLR_STAMP(12);
         lbs.flush(prm.stats, lane);
         return;
     }
@@ -533,18 +537,25 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // phase B of position nb reads its tile id from slot_tile[nb % NS]:
     // written at the end of phase A(nb), overwritten only by phase A(nb + NS)
     int na = 0, nb = 0;                                         // phases A / B done
-    for (; na < D; na++)
-        if (phaseA(na) >= ntiles) break;
+    for (; na < D; na++) {
+        const long long ja = phaseA(na);
+        if (na == 0 && tid == 0) PLR_STAMP(11);
+        if (ja >= ntiles) break;
+    }
     for (bool stop = na < D; !stop;) {
         const long long j = phaseA(na);
         phaseB(nb);
         nb++;
         if (j >= ntiles) stop = true; else na++;
     }
-    for (; nb < na; nb++) phaseB(nb);                           // drain
+    for (; nb < na; nb++) {                                     // drain
+        phaseB(nb);
+        if (nb == 0 && tid == 0) PLR_STAMP(13);
+    }
     // loader B, storer and look-back warps beyond the stop see *stop_pos
     tc_fence_before();
     named_sync(1, NC);
+    if (tid == 0) PLR_STAMP(15);
     if (warp == 0) {
         tc_fence_after();
         tmem_dealloc(tmem_base, TCOLS);
