@@ -102,6 +102,24 @@ __device__ __forceinline__ bool mbar_try_wait_sleep(uint64_t* bar, uint32_t pari
 #ifndef PLR_POLL_HINT_NS
 #define PLR_POLL_HINT_NS 0u               // waits that also poll a stop flag (a hint measured slower)
 #endif
+// Stop-aware waits (loader B, storer, look-back warps): a try_wait whose
+// phase does not complete suspends the warp for ~4 us whatever the hint
+// (0, 200, 2000 ns measured alike, profiles/r02p_small_n_trace.md), so a
+// stop set meanwhile was seen microseconds late -- the tail of every launch.
+// Poll with the non-blocking test_wait and a short sleep instead.
+#ifndef PLR_POLL_SLEEP_NS
+#define PLR_POLL_SLEEP_NS 64
+#endif
+__device__ __forceinline__ bool mbar_poll(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+    if (!ok && PLR_POLL_SLEEP_NS > 0) __nanosleep(PLR_POLL_SLEEP_NS);
+    return ok != 0;
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     while (!mbar_try_wait_sleep(bar, parity, PLR_WAIT_HINT_NS)) { }
 }

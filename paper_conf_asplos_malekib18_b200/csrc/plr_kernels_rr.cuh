@@ -207,7 +207,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 const int slot = f % NS;
                 const uint32_t par = (uint32_t)((f / NS) & 1);
                 bool stop = false;
-                while (!mbar_try_wait_sleep(&agg_bar[slot], par, PLR_POLL_HINT_NS))
+                while (!mbar_poll(&agg_bar[slot], par))
                     if (*stop_pos <= f) { stop = true; break; }
                 const long long j = stop ? ntiles : slot_tile[slot];
                 if (j >= ntiles) break;
@@ -226,9 +226,9 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 // signalled through stop_pos (phase B never runs for it)
                 const uint32_t par = (uint32_t)((t / SB) & 1);
                 bool stop = false;
-                while (!mbar_try_wait_sleep(&yfull[sb], par, PLR_POLL_HINT_NS))
+                while (!mbar_poll(&yfull[sb], par))
                     if (*stop_pos <= t) { stop = true; break; }
-                if (stop) break;
+                if (stop) { PLR_STAMP(13); break; }
                 const long long jt = store_tile[sb];
                 if (STORE && !(jt == ntiles - 1 && last_ragged)) {
                     bulk_store(prm.y + (size_t)jt * M, stB + (size_t)sb * SWL + kHalo, M * sizeof(T), pol);
@@ -258,7 +258,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         auto wait_agg = [&](int p) -> bool {                     // false at the stop
             const int slot = p % NS;
             const uint32_t par = (uint32_t)((p / NS) & 1);
-            while (!mbar_try_wait_sleep(&agg_bar[slot], par, PLR_POLL_HINT_NS))
+            while (!mbar_poll(&agg_bar[slot], par))
                 if (*stop_pos <= p) return false;
             return slot_tile[slot] < ntiles;
         };
@@ -317,6 +317,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             for (int q = 0; q < K; q++) Gi[q] = Lp[G - 1][q];
             matvec_acc<A, K>(Gi, tb.Tpow[0], Gp);              // G_J = L_{G-1} + T(G m) G_{J-1}
             publish_status<A, K, DEC>(prm.status, prm.status_mask, J, Gi, tagI, lane);
+            if (u == 0 && lane == 0) PLR_STAMP(11);
         }
         if (warp == W + 1 && lane == 0) PLR_STAMP(12);
         lbs.flush(prm.stats, lane);
@@ -539,7 +540,6 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     int na = 0, nb = 0;                                         // phases A / B done
     for (; na < D; na++) {
         const long long ja = phaseA(na);
-        if (na == 0 && tid == 0) PLR_STAMP(11);
         if (ja >= ntiles) break;
     }
     for (bool stop = na < D; !stop;) {
@@ -550,7 +550,6 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     }
     for (; nb < na; nb++) {                                     // drain
         phaseB(nb);
-        if (nb == 0 && tid == 0) PLR_STAMP(13);
     }
     // loader B, storer and look-back warps beyond the stop see *stop_pos
     tc_fence_before();

@@ -307,7 +307,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         auto wait_agg = [&](int p) -> bool {
             const int slot = p % NT;
             const uint32_t par = (uint32_t)((p / NT) & 1);
-            while (!mbar_try_wait_sleep(&agg_bar[slot], par, PLR_POLL_HINT_NS))
+            while (!mbar_poll(&agg_bar[slot], par))
                 if (*stop_pos <= p) return false;
             return slot_tile[slot] < ntiles;
         };

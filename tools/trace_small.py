@@ -10,7 +10,7 @@ import torch  # noqa: E402
 import paper_conf_asplos_malekib18_b200 as plr  # noqa: E402
 import workloads  # noqa: E402
 
-NAMES = ["init", "entry", "phaseA0_done", "lookback_warp_exit", "phaseB0_done", "storer_exit", "compute_end"]
+NAMES = ["init", "entry", "lookback_unit0_done", "lookback_warp_exit", "storer_saw_stop", "storer_exit", "compute_end"]
 for name in ["tuple2", "order3"]:
     for n in [1024, 7936 * 4, 1 << 20, 1 << 22]:
         sig = workloads.BY_NAME[name]
