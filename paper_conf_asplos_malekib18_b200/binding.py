@@ -127,6 +127,11 @@ class Plan:
                "plr_plan_create")
         self._h = h
         self._hist = None
+        self.device = None                      # CUDA device the plan's scratch lives on
+        if self.n_max > 0:
+            torch = _torch()
+            if torch.cuda.is_available():
+                self.device = torch.cuda.current_device()
 
     # ------------------------------------------------------------------
     def close(self):
@@ -172,11 +177,34 @@ class Plan:
         return out
 
     # ------------------------------------------------------------------
+    def _on_plan_device(self, *ts):
+        """Every tensor must live on the device the plan was created on."""
+        for t in ts:
+            if t is not None and t.is_cuda and self.device is not None and t.device.index != self.device:
+                raise ValueError("tensor on cuda:%d, plan created on cuda:%d" % (t.device.index, self.device))
+
     def _out(self, x, out):
         torch = _torch()
         if out is None:
             out = torch.empty_like(x)
+        elif out.numel() != x.numel():
+            raise ValueError("out has %d elements, x has %d" % (out.numel(), x.numel()))
+        self._on_plan_device(x, out)
         return out
+
+    def _hists(self, x_hist, y_hist):
+        if x_hist is not None and x_hist.numel() < self.p:
+            raise ValueError("x_hist needs the p = %d previous inputs" % self.p)
+        if y_hist is not None and y_hist.numel() < self.k:
+            raise ValueError("y_hist needs the k = %d previous outputs" % self.k)
+        self._on_plan_device(x_hist, y_hist)
+
+    @staticmethod
+    def _payload_ok(payload, nbytes=PAYLOAD_BYTES):
+        if payload.numel() * payload.element_size() < nbytes:
+            raise ValueError("payload buffer needs %d bytes" % nbytes)
+        if not payload.is_contiguous():
+            raise ValueError("payload buffer must be contiguous")
 
     def __call__(self, x, out=None, stream=None):
         """y = recurrence(x) with zero initial conditions."""
@@ -189,6 +217,7 @@ class Plan:
     def continue_(self, x, out=None, x_hist=None, y_hist=None, stream=None):
         """Continue a sequence from the p previous inputs and k previous outputs."""
         out = self._out(x, out)
+        self._hists(x_hist, y_hist)
         xh = _dev_ptr(x_hist, self.dtype) if x_hist is not None else None
         yh = _dev_ptr(y_hist, self.dtype) if y_hist is not None else None
         _check(lib.plr_execute_continue(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), x.numel(),
@@ -200,6 +229,8 @@ class Plan:
         torch = _torch()
         if payload is None:
             payload = torch.empty(PAYLOAD_BYTES, dtype=torch.uint8, device=x.device)
+        self._payload_ok(payload)
+        self._on_plan_device(x, payload)
         _check(lib.plr_reduce(self._h, _dev_ptr(x, self.dtype), x.numel(), ctypes.c_void_p(payload.data_ptr()),
                               _stream_ptr(stream)), "plr_reduce")
         return payload
@@ -208,6 +239,10 @@ class Plan:
         torch = _torch()
         if payload is None:
             payload = torch.empty(PAYLOAD_BYTES, dtype=torch.uint8, device=x.device)
+        if y.numel() != x.numel():
+            raise ValueError("y has %d elements, x has %d" % (y.numel(), x.numel()))
+        self._payload_ok(payload)
+        self._on_plan_device(x, y, payload)
         _check(lib.plr_payload_from_output(self._h, _dev_ptr(x, self.dtype), _dev_ptr(y, self.dtype), x.numel(),
                                            ctypes.c_void_p(payload.data_ptr()), _stream_ptr(stream)),
                "plr_payload_from_output")
@@ -219,6 +254,11 @@ class Plan:
         if hist is None:                        # 8 slots x_{-4..-1}, y_{-4..-1} in the plan's dtype
             hist = torch.zeros(8, dtype=torch.int32 if self.dtype == "int32" else torch.float32,
                                device=payloads.device)
+        if not 0 <= rank < world:
+            raise ValueError("rank %d outside world %d" % (rank, world))
+        self._payload_ok(payloads, world * PAYLOAD_BYTES)
+        self._payload_ok(hist, 32)
+        self._on_plan_device(payloads, hist)
         _check(lib.plr_combine(self._h, ctypes.c_void_p(payloads.data_ptr()), rank, world,
                                ctypes.c_void_p(hist.data_ptr()), _stream_ptr(stream)), "plr_combine")
         return hist
@@ -231,6 +271,8 @@ class Plan:
         return hist.raw
 
     def fixup(self, y, hist, stream=None):
+        self._payload_ok(hist, 32)
+        self._on_plan_device(y, hist)
         _check(lib.plr_fixup(self._h, _dev_ptr(y, self.dtype), y.numel(), ctypes.c_void_p(hist.data_ptr()),
                              _stream_ptr(stream)), "plr_fixup")
         return y
@@ -241,7 +283,13 @@ class Plan:
         torch = _torch()
         if y_host is None:
             y_host = torch.empty_like(x_host, pin_memory=x_host.is_pinned())
-        assert not x_host.is_cuda and not y_host.is_cuda
+        if x_host.is_cuda or y_host.is_cuda:
+            raise ValueError("execute_host takes host tensors")
+        if y_host.numel() != x_host.numel() or not x_host.is_contiguous() or not y_host.is_contiguous():
+            raise ValueError("x_host / y_host must be contiguous and of equal length")
+        want = _torch().int32 if self.dtype == "int32" else _torch().float32
+        if x_host.dtype != want or y_host.dtype != want:
+            raise TypeError("expected %s host tensors" % want)
         _check(lib.plr_execute_host(self._h, ctypes.c_void_p(x_host.data_ptr()), ctypes.c_void_p(y_host.data_ptr()),
                                     x_host.numel(), _stream_ptr(stream)), "plr_execute_host")
         return y_host

@@ -110,15 +110,40 @@ __device__ __forceinline__ bool mbar_try_wait_sleep(uint64_t* bar, uint32_t pari
 #ifndef PLR_POLL_SLEEP_NS
 #define PLR_POLL_SLEEP_NS 64
 #endif
-__device__ __forceinline__ bool mbar_poll(uint64_t* bar, uint32_t parity) {
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
     uint32_t ok;
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
         "mbarrier.test_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n\t"
         "selp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-    if (!ok && PLR_POLL_SLEEP_NS > 0) __nanosleep(PLR_POLL_SLEEP_NS);
     return ok != 0;
+}
+__device__ __forceinline__ bool mbar_poll(uint64_t* bar, uint32_t parity) {
+    const bool ok = mbar_test(bar, parity);
+    if (!ok && PLR_POLL_SLEEP_NS > 0) __nanosleep(PLR_POLL_SLEEP_NS);
+    return ok;
+}
+// Stop-aware wait of a whole warp on a phase that may never complete (a
+// pipeline position at or beyond the launch's stop): true when the phase
+// completed, false once the stop position is known to be <= pos.  While
+// tickets remain (*draining == 0) the warp suspends in try_wait and takes no
+// issue slots from the compute warps; once the loader saw the tickets run
+// out it polls (test_wait + a short sleep) so the stop is noticed at once.
+// Only for warps whose lanes all wait together (the look-back warps): a
+// suspended lane could hold back a diverged sibling lane of the producer
+// warp that the awaited arrival depends on (those lanes use mbar_poll).
+__device__ __forceinline__ bool mbar_wait_or_stop(uint64_t* bar, uint32_t parity, const volatile int* stop_pos,
+                                                  int pos, const volatile int* draining) {
+    for (;;) {
+        if (mbar_test(bar, parity)) return true;
+        if (*stop_pos <= pos) return false;
+        if (*draining) {
+            if (PLR_POLL_SLEEP_NS > 0) __nanosleep(PLR_POLL_SLEEP_NS);
+        } else if (mbar_try_wait_sleep(bar, parity, PLR_WAIT_HINT_NS)) {
+            return true;
+        }
+    }
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     while (!mbar_try_wait_sleep(bar, parity, PLR_WAIT_HINT_NS)) { }

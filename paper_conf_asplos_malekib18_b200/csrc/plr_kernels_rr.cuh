@@ -59,6 +59,7 @@ struct LayoutR {
     // ids: tileA[SA], slot_tile[NS], store_tile[SB] (long long)
     static constexpr size_t off_tmem = off_ids + (size_t)(SA + NS + SB) * 8;
     static constexpr size_t off_stop = off_tmem + 4;
+    static constexpr size_t off_drain = off_tmem + 8;                           // tickets exhausted (int)
     static constexpr size_t off_lbstat = off_tmem + 16;                         // [kMaxNL][kLbStatWords]
     static constexpr size_t bytes = off_lbstat + kMaxNL * kLbStatWords * 8;
 };
@@ -87,11 +88,9 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                              : NS * WQ * CW <= 256 ? 256 : 512;   // power-of-two allocation
     static_assert(P <= kHalo, "halo");
     static_assert(G >= 1 && G <= kMaxG && G + 1 <= NS, "look-back unit of G tiles needs G+1 slots");
-    // guard: every configuration with 2G >= NS tried on B200 hung (re-read
-    // kernel: G = 4 at NS = 8, G = 5..8 at NS = 9/10, G = 6 at NS = 12; TMEM
-    // kernel: G = 4 at NT = 7), with or without try_wait suspend hints; the
-    // cause is not identified, so such configurations do not compile
-    static_assert(2 * G < NS, "look-back unit too large for the slot ring");
+    // (NL-1) G >= NS used to hang (profiles/r02d_unit_size_hangs.txt): a
+    // look-back warp's first agg wait of its next unit ran more than one
+    // phase ahead of its slot; wait_agg now chains its waits
     static_assert(SB >= 2 && SA >= 1, "stages");
     constexpr bool DEC = false;
 
@@ -114,6 +113,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     long long* store_tile = slot_tile + NS;                     // tile id of each phase-B stage
     uint32_t* tmem_base_p = reinterpret_cast<uint32_t*>(smem + L::off_tmem);
     volatile int* stop_pos = reinterpret_cast<volatile int*>(smem + L::off_stop);
+    volatile int* draining = reinterpret_cast<volatile int*>(smem + L::off_drain);
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -137,6 +137,8 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         for (int s = 0; s < SB; s++) { mbar_init(&fullB[s], 1); mbar_init(&emptyB[s], 1); mbar_init(&yfull[s], NC); }
         for (int s = 0; s < NS; s++) { mbar_init(&agg_bar[s], 1); mbar_init(&carry_bar[s], 1); }
         *stop_pos = 1 << 30;
+        // few units per CTA (small n): every stop-aware wait polls from the start
+        *draining = (long long)((ntiles + G - 1) / G) <= 2LL * gridDim.x ? 1 : 0;
         fence_mbar_init();
     }
     if (warp == 0) tmem_alloc(tmem_base_p, TCOLS);
@@ -189,6 +191,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     const long long rel = f % G != 0 ? (long long)(atomicAdd(prm.ticket, 1ull) - tbase) : unit;
                     launch_state_advance(prm.ticket, rel, (unsigned long long)((ntiles + G - 1) / G) + gridDim.x,
                                          tbase, epoch);
+                    *draining = 1;                                  // the stop is SA..NS tiles away
                     mbar_arrive(&fullA[s]);
                     break;
                 }
@@ -255,12 +258,25 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         static_assert(NL <= kMaxNL, "look-back warps");
         const LbStats lbs{reinterpret_cast<unsigned long long*>(smem + L::off_lbstat) + (warp - W - 1) * kLbStatWords};
         lbs.init(lane);
-        auto wait_agg = [&](int p) -> bool {                     // false at the stop
-            const int slot = p % NS;
-            const uint32_t par = (uint32_t)((p / NS) & 1);
-            while (!mbar_poll(&agg_bar[slot], par))
-                if (*stop_pos <= p) return false;
-            return slot_tile[slot] < ntiles;
+        // Aggregate of pipeline position p (false at the stop).  A parity wait
+        // is exact only if the slot's previous phase (position p - NS) has
+        // completed: a barrier two phases behind reports the parity of an
+        // older phase as done (stale slot_tile / sAt: wrong unit or carry, a
+        // hang or silent corruption).  Positions complete in order and this
+        // warp saw every position <= known complete, so it first waits for
+        // known + NS (exact) until p - NS <= known.
+        int known = -1;
+        auto wait_pos = [&](int q) -> bool {
+            return mbar_wait_or_stop(&agg_bar[q % NS], (uint32_t)((q / NS) & 1), stop_pos, q, draining);
+        };
+        auto wait_agg = [&](int p) -> bool {
+            while (known < p - NS) {
+                if (!wait_pos(known + NS)) return false;
+                known += NS;
+            }
+            if (!wait_pos(p)) return false;
+            if (p > known) known = p;
+            return slot_tile[p % NS] < ntiles;
         };
         for (int u = warp - (W + 1);; u += NL) {
             const long long c_start = clock64();

@@ -144,6 +144,7 @@ struct LayoutT {
     // stop position (pipeline index of the compute warps' stop marker)
     static constexpr size_t off_tmem = off_ids + (size_t)(SL + ST + NT) * 8;
     static constexpr size_t off_stop = off_tmem + 4;
+    static constexpr size_t off_drain = off_tmem + 8;                           // tickets exhausted (int)
     static constexpr size_t off_lbstat = off_tmem + 16;                         // [kMaxNL][kLbStatWords]
     static constexpr size_t bytes = off_lbstat + kMaxNL * kLbStatWords * 8;
 };
@@ -170,11 +171,8 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     static_assert(NT >= 2 && NT * WQ * CW <= 512, "TMEM columns");
     static_assert(P <= kHalo, "halo");
     static_assert(G >= 1 && G <= kMaxG && G + 1 <= NT, "look-back unit of G tiles needs G+1 parked tiles");
-    // guard: every configuration with 2G >= NT tried on B200 hung (re-read
-    // kernel: G = 4 at NS = 8, G = 5..8 at NS = 9/10, G = 6 at NS = 12; TMEM
-    // kernel: G = 4 at NT = 7), with or without try_wait suspend hints; the
-    // cause is not identified, so such configurations do not compile
-    static_assert(2 * G < NT, "look-back unit too large for the slot ring");
+    // (NL-1) G >= NT used to hang (profiles/r02d_unit_size_hangs.txt): see
+    // wait_agg's chained waits and DESIGN.md §10
     constexpr bool DEC = false;
 
     extern __shared__ __align__(128) unsigned char smem[];
@@ -195,6 +193,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     long long* slot_tile = store_tile + ST;
     uint32_t* tmem_base_p = reinterpret_cast<uint32_t*>(smem + L::off_tmem);
     volatile int* stop_pos = reinterpret_cast<volatile int*>(smem + L::off_stop);
+    volatile int* draining = reinterpret_cast<volatile int*>(smem + L::off_drain);
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -217,6 +216,8 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         for (int s = 0; s < ST; s++) { mbar_init(&full_T[s], NC); mbar_init(&empty_T[s], 1); }
         for (int s = 0; s < NT; s++) { mbar_init(&agg_bar[s], 1); mbar_init(&carry_bar[s], 1); }
         *stop_pos = 1 << 30;
+        // few units per CTA (small n): every stop-aware wait polls from the start
+        *draining = (long long)((ntiles + G - 1) / G) <= 2LL * gridDim.x ? 1 : 0;
         fence_mbar_init();
     }
     if (warp == 0) tmem_alloc(tmem_base_p, 512);
@@ -244,6 +245,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     const long long rel = f % G != 0 ? (long long)(atomicAdd(prm.ticket, 1ull) - tbase) : unit;
                     launch_state_advance(prm.ticket, rel, (unsigned long long)((ntiles + G - 1) / G) + gridDim.x,
                                          tbase, epoch);
+                    *draining = 1;                                  // the stop is SL..NT tiles away
                     mbar_arrive(&full_L[s]);
                     break;
                 }
@@ -303,13 +305,21 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         static_assert(NL <= kMaxNL, "look-back warps");
         const LbStats lbs{reinterpret_cast<unsigned long long*>(smem + L::off_lbstat) + (warp - W - 1) * kLbStatWords};
         lbs.init(lane);
-        // wait for the aggregate of pipeline position p; false at the stop
+        // aggregate of pipeline position p (false at the stop); parity waits
+        // chained so none runs more than one phase ahead of its slot (as in
+        // plr_kernels_rr.cuh: positions <= known were seen complete)
+        int known = -1;
+        auto wait_pos = [&](int q) -> bool {
+            return mbar_wait_or_stop(&agg_bar[q % NT], (uint32_t)((q / NT) & 1), stop_pos, q, draining);
+        };
         auto wait_agg = [&](int p) -> bool {
-            const int slot = p % NT;
-            const uint32_t par = (uint32_t)((p / NT) & 1);
-            while (!mbar_poll(&agg_bar[slot], par))
-                if (*stop_pos <= p) return false;
-            return slot_tile[slot] < ntiles;
+            while (known < p - NT) {
+                if (!wait_pos(known + NT)) return false;
+                known += NT;
+            }
+            if (!wait_pos(p)) return false;
+            if (p > known) known = p;
+            return slot_tile[p % NT] < ntiles;
         };
         for (int u = warp - (W + 1);; u += NL) {               // NL look-back warps take turns
             const long long c_start = clock64();
@@ -559,9 +569,12 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     for (; nb < na; nb++) phaseB(nb);                           // drain
     // stop markers: the storer, and look-back warps waiting beyond the stop
     {
-        // no wait for the stage: only its id slot is written, and the storer
-        // (which is at tile >= nb-2) has long read the previous id of it
+        // wait for the stage as phase B of position nb would: with STORE =
+        // false the storer releases stages at once, so it may not have
+        // consumed position nb - ST yet; arriving early would complete
+        // full_T[sT] a phase ahead of its parity wait (a hang)
         const int sT = nb % ST;
+        mbar_wait(&empty_T[sT], (uint32_t)(((nb / ST) & 1) ^ 1));
         if (tid == 0) store_tile[sT] = ntiles;
         mbar_arrive(&full_T[sT]);
     }

@@ -6,6 +6,7 @@
 #include "plr_kernels_tmem.cuh"
 #include "plr_kernels_rr.cuh"
 #include "plr_launch.h"
+#include <atomic>
 #include <type_traits>
 
 namespace plr {
@@ -60,13 +61,24 @@ namespace inst {
 #define PLR_GEN_TMEM (PLR_GEN_KIND != 0)
 // re-read kernel (measured r01r-r01u): X = 31, W = 8 (tile 7936), 3 look-back
 // warps, 2 HBM load stages, 5 L2 re-read / store stages, phase-B lag 8 tiles,
-// look-back units of 4 tiles (G >= 5 hung at NS = 9: not used)
+// look-back units of 4 tiles (G >= 5 hung at NS = 9 before the chained agg
+// waits of DESIGN.md §10)
 #ifndef PLR_RR_X
 #define PLR_RR_X 31
+#endif
+#ifndef PLR_RR_W
 #define PLR_RR_W 8
+#endif
+#ifndef PLR_RR_NL
 #define PLR_RR_NL 3
+#endif
+#ifndef PLR_RR_SA
 #define PLR_RR_SA 2         // phase-A (HBM) load stages
+#endif
+#ifndef PLR_RR_SB
 #define PLR_RR_SB 5         // phase-B (L2 re-read + y store) stages
+#endif
+#ifndef PLR_RR_NS
 #define PLR_RR_NS 9         // slots: phase B lags phase A by NS-1 tiles (L2 reuse distance)
 #endif
 #ifndef PLR_RR_G
@@ -74,9 +86,17 @@ namespace inst {
 #endif
 #ifndef PLR_TM_X
 #define PLR_TM_X 15
+#endif
+#ifndef PLR_TM_W
 #define PLR_TM_W 16
+#endif
+#ifndef PLR_TM_NL
 #define PLR_TM_NL 2
+#endif
+#ifndef PLR_TM_SL
 #define PLR_TM_SL 3
+#endif
+#ifndef PLR_TM_ST
 #define PLR_TM_ST 3
 #endif
 #ifndef PLR_TM_G
@@ -135,11 +155,16 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
         smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
         threads = (C::W + 1 + C::NL) * 32;
     }
-    static bool configured = false;
-    if (!configured) {
+    // the > 48 KB dynamic shared memory opt-in is a per-device (context)
+    // attribute: one bit per device, set once (racing sets are idempotent)
+    static std::atomic<unsigned long long> configured{0};
+    int dev = 0;
+    if (cudaError_t e = cudaGetDevice(&dev); e != cudaSuccess) return e;
+    const unsigned long long bit = 1ull << (dev & 63);
+    if (!(configured.load(std::memory_order_acquire) & bit)) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        configured = true;
+        configured.fetch_or(bit, std::memory_order_acq_rel);
     }
     if (la.occupancy_out != nullptr) {  // occupancy query: report CTAs/SM, do not launch
         cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, threads, smem);

@@ -284,8 +284,10 @@ def _stream_check(plr_mod, torch, sig, n, seed, seg=1 << 25):
     torch.cuda.empty_cache()
 
 
-@pytest.mark.parametrize("name", ["tuple2", "tuple3", "order2", "order3", "lp1", "lp2", "hp2", "prefix"])
+@pytest.mark.parametrize("name", [s.name for s in workloads.TABLE1])
 def test_full_size_parity(cuda_plr, name):
+    """Every Table-1 row at exactly n = 2^30, every
+    output element compared."""
     import torch
     sig = workloads.BY_NAME[name]
     _stream_check(cuda_plr, torch, sig, FULL, workloads.seed_for(2))
@@ -294,3 +296,67 @@ def test_full_size_parity(cuda_plr, name):
 def test_full_size_ragged(cuda_plr):
     import torch
     _stream_check(cuda_plr, torch, workloads.BY_NAME["hp3"], FULL - 12345, workloads.seed_for(6))
+
+
+# ------------------------------------------------------------ ablation -----
+ABLATIONS = {"generic": ("PLR_FORCE_GENERIC", "1"), "no_constsig": ("PLR_NO_CONSTSIG", "1")}
+
+
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+@pytest.mark.parametrize("mode", sorted(ABLATIONS))
+def test_ablation_modes_parity(cuda_plr, sig, mode, monkeypatch):
+    """The Fig. 10 analogue (tools/ablation.py) times kernels
+    with the class specialisations off (PLR_FORCE_GENERIC=1: DECAY rows on
+    the generic multi-tile look-back, no compile-time tables) or the
+    compile-time signature tables off (PLR_NO_CONSTSIG=1).  Those kernels
+    must meet the same parity bar as the shipped ones."""
+    import torch
+    var, val = ABLATIONS[mode]
+    monkeypatch.setenv(var, val)
+    probe = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 10)
+    m = probe.info["tile_elems"]
+    if mode == "generic":
+        assert probe.info["kernel_kind"] != 0 and probe.info["const_sig"] == 0
+    else:
+        assert probe.info["const_sig"] == 0
+    probe.close()
+    sizes = [1, 5, m - 1, m + 1, 7 * m + 3, 33 * m + 5, (1 << 20) + 12345]
+    x_all = workloads.host_input(max(sizes), sig.dtype, workloads.seed_for(9))
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=max(sizes))
+    for n in sizes:
+        x = x_all[:n].copy()
+        y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+        check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s %s n=%d" % (sig.name, mode, n))
+    xa = workloads.structured_input("alternating", 7 * m + 123, sig.dtype)
+    y = plan(torch.from_numpy(xa).cuda()).cpu().numpy()
+    check(y, oracle.recurrence(xa, sig.a, sig.b, sig.dtype), sig.dtype, "%s %s alternating" % (sig.name, mode))
+    plan.close()
+
+
+# ------------------------------------------------------------ determinism --
+@pytest.mark.parametrize("sig", [s for s in workloads.TABLE1 if s.dtype == "float32"], ids=lambda s: s.name)
+def test_decay_bitwise_repeatable(cuda_plr, sig):
+    """DECAY float results are bitwise repeatable, because
+    T(m) = 0 makes the look-back a single hop (the carry entering a tile
+    never depends on which predecessor happened to be inclusive).  Repeated
+    launches, with and without a concurrent memory-bound kernel on another
+    stream perturbing the tile-to-CTA schedule, give identical bits."""
+    import torch
+    n = (1 << 24) + 777
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    assert plan.info["cls"] == "DECAY"
+    xd = workloads.device_input(n, sig.dtype, workloads.seed_for(10))
+    first = plan(xd).cpu().numpy().view(np.uint32)
+    noise_a = torch.empty(1 << 27, dtype=torch.float32, device="cuda")
+    noise_b = torch.empty_like(noise_a)
+    side = torch.cuda.Stream()
+    for t in range(6):
+        if t % 2:
+            with torch.cuda.stream(side):
+                for _ in range(3):
+                    noise_b.copy_(noise_a)
+        y = plan(xd).cpu().numpy().view(np.uint32)
+        torch.cuda.synchronize()
+        assert np.array_equal(y, first), "%s: run %d differs bitwise in %d elements" % (
+            sig.name, t, int(np.count_nonzero(y != first)))
+    plan.close()

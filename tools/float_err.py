@@ -1,0 +1,64 @@
+"""Worst relative error per float Table-1 row: every
+output of the shipped kernel at n = 2^30 (seeded U[-1,1), streamed oracle
+comparison) and on the worked example's alternating input (-1)^i (i+3)
+ at n = 7*3840+123, against the fp64 oracle; bar 1e-4 (north_star).
+Prints a markdown table."""
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import oracle  # noqa: E402
+import paper_conf_asplos_malekib18_b200 as plr  # noqa: E402
+import workloads  # noqa: E402
+
+
+def rel(y, ref):
+    e = np.abs(y.astype(np.float64) - ref) / np.maximum(1.0, np.abs(ref))
+    i = int(np.argmax(e))
+    return float(e[i]), i
+
+
+def full(sig, n, seed, seg=1 << 25):
+    plan = plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    xd = workloads.device_input(n, sig.dtype, seed)
+    yd = plan(xd)
+    torch.cuda.synchronize()
+    xh = yh = None
+    worst, where = 0.0, -1
+    for s in range(0, n, seg):
+        e = min(n, s + seg)
+        x = xd[s:e].cpu().numpy()
+        y = yd[s:e].cpu().numpy()
+        ref = oracle.recurrence(x, sig.a, sig.b, sig.dtype, x_hist=xh, y_hist=yh)
+        w, i = rel(y, ref)
+        if w > worst:
+            worst, where = w, s + i
+        xh = x[len(x) - sig.p:] if sig.p else None
+        yh = ref[len(ref) - sig.k:]
+    info = plan.info
+    plan.close()
+    del xd, yd
+    torch.cuda.empty_cache()
+    return worst, where, info
+
+
+n = int(sys.argv[1]) if len(sys.argv) > 1 else 1 << 30
+print("| row | kernel | acc | U[-1,1) n=%d worst rel err | at index | alternating ±(i+3) n=27003 | bar |" % n)
+print("|---|---|---|---|---|---|---|")
+for sig in workloads.TABLE1:
+    if sig.dtype != "float32":
+        continue
+    t0 = time.time()
+    w, i, info = full(sig, n, workloads.seed_for(2))
+    xa = workloads.structured_input("alternating", 7 * 3840 + 123, "float32")
+    pa = plr.Plan(sig.a, sig.b, sig.dtype, n_max=len(xa))
+    ya = pa(torch.from_numpy(xa).cuda()).cpu().numpy()
+    wa, _ = rel(ya, oracle.recurrence(xa, sig.a, sig.b, sig.dtype))
+    pa.close()
+    print("| %s | %s | %s | %.3g | %d | %.3g | 1e-4 |" % (
+        sig.name, info.get("kernel_kind"), info.get("acc", "?"), w, i, wa), flush=True)
+    sys.stderr.write("%s %.1fs\n" % (sig.name, time.time() - t0))

@@ -104,12 +104,9 @@ def structured_input(kind: str, n: int, dtype: str) -> np.ndarray:
         if n:
             x[0] = 1
         return x
-    if kind == "alternating":
+    if kind == "alternating":          # the worked example's input pattern (-1)^i (i+3)
         i = np.arange(n, dtype=np.int64)
-        if dtype == "int32":           # the worked example's input pattern
-            v = np.where(i % 2 == 0, 1, -1) * (i + 3)
-        else:                          # unit amplitude: float workloads live in [-1, 1)
-            v = np.where(i % 2 == 0, 1.0, -1.0)
+        v = np.where(i % 2 == 0, 1, -1) * (i + 3)
         return v.astype(npdt)
     if kind == "extremes":
         v = np.array([2 ** 31 - 1, -(2 ** 31), -1, 1], dtype=np.int64)
