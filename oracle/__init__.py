@@ -55,6 +55,7 @@ def _load():
             I = ctypes.c_int
             lib.oracle_eq1_i32.argtypes = [P, P, I64, P, I, P, I, P, P]
             lib.oracle_eq1_f64.argtypes = [P, P, I64, P, I, P, I, P, P]
+            lib.oracle_eq1_f64_dd.argtypes = [P, P, I64, P, I, P, I]
             lib.oracle_factor_lists_i32.argtypes = [P, I, I64, P]
             lib.oracle_factor_lists_f64.argtypes = [P, I, I64, P]
             lib.oracle_phase1_i32.argtypes = [P, I64, P, I, I64, P, I64, P]
@@ -115,6 +116,32 @@ def recurrence(x, a, b, dtype: str, x_hist=None, y_hist=None, exact_coeffs: bool
         assert xh is None or xh.shape[0] == p
         assert yh is None or yh.shape[0] == k
         lib.oracle_eq1_f64(_ptr(x), _ptr(y), x.shape[0], _ptr(af), p, _ptr(bf), k, _ptr(xh), _ptr(yh))
+        return y
+    raise ValueError(dtype)
+
+
+def cascade(x, stages, dtype: str) -> np.ndarray:
+    """A cascade of signatures ("inputs that consist of multiple signatures",
+    P:1851-1852; filters applied one after the other): stage s
+    evaluates Eq. (1) with its own (a_s : b_s) on the previous stage's
+    output, zero initial conditions.  int32: every stage in Z/2^32; float32:
+    every stage in fp64 with its fp32-rounded coefficients, stage outputs
+    not rounded in between.  stages: sequence of (a, b) pairs (b may be
+    empty: a feed-forward stage)."""
+    lib = _load()
+    if dtype == "int32":
+        y = np.ascontiguousarray(x, dtype=np.int32)
+        for a, b in stages:
+            y = recurrence(y, a, b, "int32")
+        return y
+    if dtype == "float32":
+        y = np.ascontiguousarray(x, dtype=np.float32).astype(np.float64)
+        for a, b in stages:
+            af, bf = f32c(a), f32c(b)
+            out = np.empty_like(y)
+            lib.oracle_eq1_f64_dd(_ptr(y), _ptr(out), y.shape[0], _ptr(af), len(a) - 1,
+                                  _ptr(bf) if len(bf) else None, len(bf))
+            y = out
         return y
     raise ValueError(dtype)
 

@@ -119,6 +119,25 @@ void oracle_eq1_f64(const float* x, double* y, int64_t n,
     }
 }
 
+/* Eq. (1) in fp64 over an fp64 input: one stage of a cascade, whose input is
+ * the previous stage's (unrounded) output.  A cascade of filters feeds the
+ * output of one filter into the next (a higher-order filter
+ * decomposed into several lower-order ones; "inputs that consist of multiple
+ * signatures").  Same order of terms as oracle_eq1_f64, zero
+ * initial conditions. */
+void oracle_eq1_f64_dd(const double* x, double* y, int64_t n,
+                       const double* a, int p, const double* b, int k)
+{
+    for (int64_t i = 0; i < n; i++) {
+        double acc = 0.0;
+        for (int j = 0; j <= p; j++)
+            if (i - j >= 0) acc += a[j] * x[i - j];
+        for (int j = 1; j <= k; j++)
+            if (i - j >= 0) acc += b[j - 1] * y[i - j];
+        y[i] = acc;
+    }
+}
+
 /* ---------------------------------------------------------------------- */
 /* Correction-factor lists (Sec. 2.1)                            */
 /* ---------------------------------------------------------------------- */

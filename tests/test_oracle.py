@@ -289,3 +289,51 @@ def test_zero_length_and_short():
                                  sig.a, sig.b, sig.dtype).shape == (0,)
     y = oracle.recurrence(np.array([5, 7], np.int32), (1,), (3, -3, 1), "int32")
     assert y.tolist() == [5, 7 + 15]
+
+
+# ---------------------------------------------------------------- cascade --
+def test_cascade_of_prefix_sums_is_binomial():
+    """Three cascaded prefix sums (1: 1) on ones give C(i+3, 3) mod 2^32 --
+    the 3rd-order prefix sum (binomial signatures) as a
+    multi-signature input."""
+    n = 3000
+    i = np.arange(n, dtype=object)
+    y = oracle.cascade(np.ones(n, np.int32), [((1,), (1,))] * 3, "int32")
+    expect = [wrap32(int(v)) for v in (i + 1) * (i + 2) * (i + 3) // 6]
+    assert y.tolist() == expect
+
+
+def test_cascade_int_matches_composed_signature_bitwise():
+    """Z/2^32 is a ring: a cascade equals the single signature with the
+    multiplied polynomials, bit for bit (full-range inputs, wraparound)."""
+    x = workloads.host_input(5000, "int32", 3)
+    y = oracle.cascade(x, [((3, -1), (0, 1)), ((1,), (2, -1))], "int32")
+    # (3 - z^-1) / ((1 - z^-2)(1 - 2 z^-1 + z^-2)) = (3, -1 : 2, 0, -2, 1)
+    assert np.array_equal(y, oracle.recurrence(x, (3, -1), (2, 0, -2, 1), "int32"))
+
+
+def test_cascade_lp1_twice_impulse_closed_form():
+    """(0.2: 0.8) twice: impulse response 0.04 (i+1) 0.8^i (the LP2 row's
+    closed form, with the fp32-rounded coefficients)."""
+    n = 300
+    x = np.zeros(n, np.float32)
+    x[0] = 1
+    y = oracle.cascade(x, [((0.2,), (0.8,))] * 2, "float32")
+    a, c = float(np.float32(0.2)), float(np.float32(0.8))
+    i = np.arange(n)
+    np.testing.assert_allclose(y, a * a * (i + 1) * c ** i, rtol=1e-12, atol=0)
+
+
+def test_cascade_float_matches_scipy_composed():
+    """Stage by stage (oracle) vs scipy.signal.lfilter with the convolved
+    numerator and denominator polynomials of the same fp32-rounded stages."""
+    signal = pytest.importorskip("scipy.signal")
+    stages = [((0.9, -0.9), (0.8,)), ((0.9, -0.9), (0.8,)), ((0.04,), (1.6, -0.64))]
+    x = workloads.host_input(20000, "float32", 4)
+    num, den = np.array([1.0]), np.array([1.0])
+    for a, b in stages:
+        num = np.convolve(num, oracle.f32c(a))
+        den = np.convolve(den, np.concatenate([[1.0], -oracle.f32c(b)]))
+    ref = signal.lfilter(num, den, x.astype(np.float64))
+    y = oracle.cascade(x, stages, "float32")
+    np.testing.assert_allclose(y, ref, rtol=1e-9, atol=1e-12)
