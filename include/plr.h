@@ -50,7 +50,7 @@
 extern "C" {
 #endif
 
-#define PLR_ABI_VERSION 2
+#define PLR_ABI_VERSION 3
 #define PLR_MAX_K 4            /* maximum order k supported by the kernels      */
 #define PLR_MAX_P 3            /* maximum feed-forward order p                  */
 #define PLR_PAYLOAD_BYTES 64   /* one rank's end-state record, see plr_reduce   */
@@ -102,6 +102,10 @@ typedef struct {
     int tiles_per_unit;        /* G: consecutive tiles per ticket / status record / look-back */
     int kernel_kind;           /* scan kernel: 0 DECAY single-hop pipeline, 1 TMEM-parking,
                                   2 L2 re-read (generic classes), 3 generic smem pipeline */
+    int acc_bits;              /* accumulation of the chunk recurrence and carries: 32 (the
+                                  data type) or 64 (fp64, reading R16)       */
+    double cond_bound;         /* float: the planner's a-priori error bound of fp32
+                                  accumulation relative to the output scale (R16); 0 int */
 } plr_plan_info;
 
 /* Create a plan.  a[0..p] = (a0, a-1, ..., a-p) (p = feed-forward order, so
@@ -119,6 +123,28 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
                            plr_dtype dtype, size_t n_max);
 plr_status plr_plan_destroy(plr_plan* plan);
 plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info);
+
+/* A cascade of `nstages` signatures evaluated in ONE pass ("inputs that
+ * consist of multiple signatures"; a higher-order filter as
+ * several lower-order ones).  Stage s is (a_s : b_s) with p[s]+1
+ * feed-forward and k[s] feedback coefficients (k[s] = 0: a pure map stage),
+ * packed stage after stage in a[] and b[].  The planner combines the stages
+ * by multiplying their z-transforms (numerators A_s(z) and denominators
+ * 1 - sum_j b_{s,j} z^-j) -- the combination the paper leaves to the user,
+ * offline -- and plans the resulting single signature: one read
+ * and one write of the data instead of one per stage.  PLR_INT32 combines in
+ * Z/2^32 (bit-exact: a ring homomorphism); PLR_FLOAT32 combines in fp64 the
+ * fp32-rounded stage coefficients.  Each stage is checked like a signature
+ * (last coefficients nonzero); the combination must have k >= 1,
+ * k <= PLR_MAX_K and p <= PLR_MAX_P (PLR_ERR_SIZE). */
+plr_status plr_plan_create_cascade(plr_plan** out, int nstages, const double* a, const int* p,
+                                   const double* b, const int* k, plr_dtype dtype, size_t n_max);
+
+/* The signature a plan evaluates (for a cascade: the combined one), as the
+ * kernels use it: a[0..p] (a0, a-1, ..., a-p) and b[0..k-1] (b-1, ..., b-k);
+ * int32 coefficients as their residues in [0, 2^32), float32 ones rounded to
+ * fp32.  Host memory (PLR_MAX_P+1 and PLR_MAX_K doubles suffice). */
+plr_status plr_plan_get_signature(const plr_plan* plan, double* a, double* b);
 
 /* Planner introspection (tests): the correction-factor lists of Sec. 2.1 as
  * the kernels use them.  out receives k rows of (k + m) values (the seed in
@@ -180,7 +206,9 @@ plr_status plr_fixup(plr_plan* plan, void* y, size_t n, const void* hist, void* 
 
 /* One segment of a sequence sharded over `world` ranks (rank r holds the
  * r-th contiguous segment; n_local may differ per rank).  `comm` is an
- * ncclComm_t from plr_nccl_comm_init.  One ncclAllGather of
+ * ncclComm_t from plr_nccl_comm_init (a 1-rank communicator is valid and
+ * takes the same NCCL path; comm may be NULL only when world == 1, which
+ * copies the payload instead of gathering it).  One ncclAllGather of
  * PLR_PAYLOAD_BYTES per rank over NVLink/NVSwitch; no other collective.
  * DECAY: local pass, allgather, sparse fixup (2n traffic).  Others:
  * reduce-only pass, allgather, seeded single pass (3n traffic). */

@@ -22,6 +22,8 @@ _st = ctypes.c_int
 
 _SIGS = {
     "plr_plan_create": ([ctypes.POINTER(_P), _P, _I, _P, _I, _I, _S], _st),
+    "plr_plan_create_cascade": ([ctypes.POINTER(_P), _I, _P, _P, _P, _P, _I, _S], _st),
+    "plr_plan_get_signature": ([_P, _P, _P], _st),
     "plr_plan_destroy": ([_P], _st),
     "plr_plan_get_info": ([_P, _P], _st),
     "plr_plan_factor_lists": ([_P, ctypes.c_int64, _P], _st),
@@ -58,7 +60,7 @@ class PlanInfo(ctypes.Structure):
                 ("threads_per_cta", _I), ("tile_elems", _I), ("stages", _I), ("decay_len", ctypes.c_int64),
                 ("fixup_len", ctypes.c_int64), ("n_max", _S), ("scratch_bytes", _S), ("ctas_per_sm", _I),
                 ("num_sms", _I), ("const_sig", _I),
-                ("tiles_per_unit", _I), ("kernel_kind", _I)]
+                ("tiles_per_unit", _I), ("kernel_kind", _I), ("acc_bits", _I), ("cond_bound", ctypes.c_double)]
 
 
 class PLRError(RuntimeError):
@@ -111,20 +113,39 @@ def shard_bounds(n_total: int, world: int, rank: int):
 class Plan:
     """A planned recurrence (signature a : b) for one dtype and up to n_max elements."""
 
-    def __init__(self, a, b, dtype: str = "int32", n_max: int = 1 << 30):
+    def __init__(self, a, b, dtype: str = "int32", n_max: int = 1 << 30, _stages=None):
         if dtype not in _DTYPES:
             raise ValueError("dtype must be 'int32' or 'float32'")
-        self.a = tuple(float(v) for v in a)
-        self.b = tuple(float(v) for v in b)
         self.dtype = dtype
+        self.n_max = int(n_max)
+        self.stages = None
+        h = _P()
+        if _stages is None:
+            self.a = tuple(float(v) for v in a)
+            self.b = tuple(float(v) for v in b)
+            arr_a = (ctypes.c_double * len(self.a))(*self.a)
+            arr_b = (ctypes.c_double * max(1, len(self.b)))(*self.b)
+            _check(lib.plr_plan_create(ctypes.byref(h), arr_a, len(self.a) - 1, arr_b, len(self.b), _DTYPES[dtype],
+                                       self.n_max), "plr_plan_create")
+        else:
+            self.stages = tuple((tuple(float(v) for v in sa), tuple(float(v) for v in sb)) for sa, sb in _stages)
+            fa = [v for sa, _ in self.stages for v in sa]
+            fb = [v for _, sb in self.stages for v in sb]
+            arr_a = (ctypes.c_double * max(1, len(fa)))(*fa)
+            arr_b = (ctypes.c_double * max(1, len(fb)))(*fb)
+            ps = (ctypes.c_int * len(self.stages))(*[len(sa) - 1 for sa, _ in self.stages])
+            ks = (ctypes.c_int * len(self.stages))(*[len(sb) for _, sb in self.stages])
+            _check(lib.plr_plan_create_cascade(ctypes.byref(h), len(self.stages), arr_a, ps, arr_b, ks,
+                                               _DTYPES[dtype], self.n_max), "plr_plan_create_cascade")
+            ca = (ctypes.c_double * 8)()
+            cb = (ctypes.c_double * 8)()
+            _check(lib.plr_plan_get_signature(h, ca, cb), "plr_plan_get_signature")
+            pi = PlanInfo()
+            _check(lib.plr_plan_get_info(h, ctypes.byref(pi)), "plr_plan_get_info")
+            self.a = tuple(ca[j] for j in range(pi.p + 1))
+            self.b = tuple(cb[j] for j in range(pi.k))
         self.p = len(self.a) - 1
         self.k = len(self.b)
-        self.n_max = int(n_max)
-        arr_a = (ctypes.c_double * len(self.a))(*self.a)
-        arr_b = (ctypes.c_double * max(1, len(self.b)))(*self.b)
-        h = _P()
-        _check(lib.plr_plan_create(ctypes.byref(h), arr_a, self.p, arr_b, self.k, _DTYPES[dtype], self.n_max),
-               "plr_plan_create")
         self._h = h
         self._hist = None
         self.device = None                      # CUDA device the plan's scratch lives on
@@ -132,6 +153,20 @@ class Plan:
             torch = _torch()
             if torch.cuda.is_available():
                 self.device = torch.cuda.current_device()
+
+    @classmethod
+    def cascade(cls, stages, dtype: str = "int32", n_max: int = 1 << 30) -> "Plan":
+        """One-pass plan of a cascade of signatures [(a_1, b_1), (a_2, b_2), ...]
+        (plr_plan_create_cascade: the stages' z-transforms multiplied by the
+        planner)."""
+        return cls(None, None, dtype, n_max, _stages=stages)
+
+    def signature(self):
+        """(a, b) as the kernels use them (int32 residues in [0, 2^32), fp32 roundings)."""
+        ca = (ctypes.c_double * 8)()
+        cb = (ctypes.c_double * 8)()
+        _check(lib.plr_plan_get_signature(self._h, ca, cb), "plr_plan_get_signature")
+        return tuple(ca[j] for j in range(self.p + 1)), tuple(cb[j] for j in range(self.k))
 
     # ------------------------------------------------------------------
     def close(self):

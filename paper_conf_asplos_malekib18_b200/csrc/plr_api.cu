@@ -8,6 +8,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <vector>
+#include <cmath>
 
 #include "plr_internal.h"
 #include "plr_launch.h"
@@ -44,6 +46,8 @@ struct plr_plan {
     unsigned long long* d_status = nullptr;
     uint32_t epoch = 0;                 // host count of launches since the last reset (overflow guard)
     void* d_lane = nullptr;
+    void* d_lane_s = nullptr;           // lane table T(X_s l) of the small-n kernel
+    size_t small_max = 0;               // n <= small_max: the small-n kernel (plr_kernels_small.cuh)
     float* d_fix = nullptr;
     bool dirty = false;
     bool sig_kernel = false;            // launch the compile-time signature kernel (pt.sig_id)
@@ -75,6 +79,14 @@ static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 static uint64_t unit1_waves() {
     const char* e = std::getenv("PLR_UNIT1_WAVES");
     return e != nullptr ? (uint64_t)std::strtoull(e, nullptr, 10) : (uint64_t)1;
+}
+
+// Sizes up to this many elements run the small-n kernel (one CTA per tile,
+// no pipeline, profiles/*_sweep.md); PLR_SMALL_MAX
+// overrides it at plan creation (0: never).
+static size_t small_max_default() {
+    const char* e = std::getenv("PLR_SMALL_MAX");
+    return e != nullptr ? (size_t)std::strtoull(e, nullptr, 10) : ((size_t)1 << 22);
 }
 
 // ============================================================ helpers =====
@@ -223,6 +235,35 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
                          const void* y_hist, void* y_tail, bool store, cudaStream_t stream) {
     if (n == 0) return PLR_OK;
     if (n > plan->n_max) return fail(PLR_ERR_SIZE, "n exceeds the plan's n_max");
+    if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
+        CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, stream), "status reset");
+        CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, kTicketBytes, stream), "ticket reset");
+        plan->epoch = 0;
+        plan->dirty = false;
+    }
+    if (n <= plan->small_max) {                 // small n: one CTA per tile, no pipeline
+        const uint64_t ms = (uint64_t)plan->pt.geo_s.tile();
+        plan->epoch++;
+        LaunchArgs la;
+        la.x = x; la.y = store ? y : nullptr; la.n = n; la.ntiles = (n + ms - 1) / ms;
+        la.ticket = plan->d_ticket;
+        la.status = plan->d_status;
+        la.status_mask = plan->status_slots - 1;
+        la.decay = plan->pt.decay_s;
+        la.dec_mask = plan->pt.dec_mask_s;
+        la.x_hist = x_hist; la.y_hist = y_hist; la.y_tail = y_tail;
+        la.lane_T = plan->d_lane_s;
+        la.stats = plan->d_stats;
+        la.grid = (int)la.ntiles;
+        la.store = store;
+        la.stream = stream;
+        cudaError_t e = launch_small(plan->pt, la);
+        if (e != cudaSuccess) {
+            plan->dirty = true;
+            return cuda_fail(e, "small-n kernel launch");
+        }
+        return PLR_OK;
+    }
     const uint64_t m = (uint64_t)plan->pt.geo.tile();
     const uint64_t ntiles = (n + m - 1) / m;
     // tiles per ticket (look-back unit).  Small n: units of one tile, so the
@@ -232,12 +273,6 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     const bool unit1 = plan->pt.geo.G > 1 && ntiles < unit1_waves() * grid_max * (uint64_t)plan->pt.geo.G;
     const uint64_t G = unit1 ? 1 : (uint64_t)plan->pt.geo.G;
     const uint64_t nunits = (ntiles + G - 1) / G;
-    if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
-        CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, stream), "status reset");
-        CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, kTicketBytes, stream), "ticket reset");
-        plan->epoch = 0;
-        plan->dirty = false;
-    }
     plan->epoch++;
     const uint64_t grid = std::min<uint64_t>(nunits, grid_max);
     LaunchArgs la;
@@ -305,6 +340,7 @@ plr_status plr_plan_destroy(plr_plan* plan) {
     cudaFree(plan->d_ticket);
     cudaFree(plan->d_status);
     cudaFree(plan->d_lane);
+    cudaFree(plan->d_lane_s);
     cudaFree(plan->d_fix);
     cudaFree(plan->d_send);
     cudaFree(plan->d_recv);
@@ -347,6 +383,7 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
         st = plan_tables(a, p, b, k, dtype, class_geometry(false, k), &plan->pt, &why);
         if (st == PLR_OK && force_generic) {
             plan->pt.decay_flag = 0;
+            plan->pt.decay_s = 0;                              // the small-n kernel's one-hop look-back too
             plan->pt.acc64 = dtype == PLR_FLOAT32 ? 1 : 0;   // generic float kernels accumulate in fp64
         }
     }
@@ -377,8 +414,12 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
         return bail(e, "SM count");
     if ((e = scan_occupancy(plan->pt, &plan->ctas_per_sm)) != cudaSuccess) return bail(e, "occupancy");
     if (plan->ctas_per_sm < 1) { plr_plan_destroy(plan); return fail(PLR_ERR_CUDA, "kernel does not fit on an SM"); }
-    const uint64_t m = (uint64_t)plan->pt.geo.tile();
+    int small_ctas = 0;
+    if ((e = small_occupancy(plan->pt, &small_ctas)) != cudaSuccess) return bail(e, "occupancy (small-n)");
+    plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default()) : 0;
+    const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
+    plan->max_tiles = std::max<uint64_t>(plan->max_tiles, (plan->small_max + ms - 1) / ms);   // status slots cover both
     if (plan->max_tiles > (1ull << 31)) { plr_plan_destroy(plan); return fail(PLR_ERR_SIZE, "n_max too large"); }
     plan->status_slots = 1;
     while (plan->status_slots < plan->max_tiles) plan->status_slots <<= 1;
@@ -392,6 +433,10 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     const void* lane_src = dtype == PLR_INT32 ? (const void*)plan->pt.lane_i
                          : acc64 ? (const void*)plan->pt.lane_d : (const void*)plan->pt.lane_f;
     if ((e = cudaMemcpy(plan->d_lane, lane_src, lane_bytes, cudaMemcpyHostToDevice)) != cudaSuccess) return bail(e, "copy lane table");
+    if ((e = cudaMalloc(&plan->d_lane_s, lane_bytes)) != cudaSuccess) return bail(e, "alloc lane table");
+    const void* lane_s = dtype == PLR_INT32 ? (const void*)plan->pt.lane_is
+                       : acc64 ? (const void*)plan->pt.lane_ds : (const void*)plan->pt.lane_fs;
+    if ((e = cudaMemcpy(plan->d_lane_s, lane_s, lane_bytes, cudaMemcpyHostToDevice)) != cudaSuccess) return bail(e, "copy lane table");
     if (plan->pt.cls == PLR_CLASS_DECAY && plan->pt.fixup_len > 0) {
         const size_t fb = (size_t)plan->pt.fixup_len * kAug * 4;
         if ((e = cudaMalloc(&plan->d_fix, fb)) != cudaSuccess) return bail(e, "alloc fixup table");
@@ -405,6 +450,70 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     }
     if ((e = cudaMemset(plan->d_hist, 0, 64)) != cudaSuccess) return bail(e, "memset hist");
     *out = plan;
+    return PLR_OK;
+}
+
+plr_status plr_plan_create_cascade(plr_plan** out, int nstages, const double* a, const int* p, const double* b,
+                                   const int* k, plr_dtype dtype, size_t n_max) {
+    if (out == nullptr) return fail(PLR_ERR_INVALID_ARG, "null out");
+    *out = nullptr;
+    if (nstages < 1 || a == nullptr || p == nullptr || k == nullptr) return fail(PLR_ERR_INVALID_ARG, "bad stage list");
+    if (dtype != PLR_INT32 && dtype != PLR_FLOAT32) return fail(PLR_ERR_DTYPE, "dtype must be PLR_INT32 or PLR_FLOAT32");
+    // numerator N(z) and denominator D(z) = 1 - sum_j b_j z^-j, multiplied
+    // stage by stage: Z/2^32 (uint64 wrapped) or fp64
+    constexpr int kCap = 64;
+    std::vector<uint64_t> Nu(1, 1), Du(1, 1);
+    std::vector<double> Nd(1, 1.0), Dd(1, 1.0);
+    const double* ap = a;
+    const double* bp = b;
+    for (int s = 0; s < nstages; s++) {
+        const int ps = p[s], ks = k[s];
+        if (ps < 0 || ks < 0 || ps >= kCap || ks >= kCap) return fail(PLR_ERR_SIGNATURE, "bad stage order");
+        if (ks > 0 && bp == nullptr) return fail(PLR_ERR_INVALID_ARG, "null b");
+        for (int j = 0; j <= ps; j++)
+            if (!std::isfinite(ap[j])) return fail(PLR_ERR_SIGNATURE, "non-finite coefficient");
+        for (int j = 0; j < ks; j++)
+            if (!std::isfinite(bp[j])) return fail(PLR_ERR_SIGNATURE, "non-finite coefficient");
+        if (ap[ps] == 0.0 || (ks > 0 && bp[ks - 1] == 0.0))
+            return fail(PLR_ERR_SIGNATURE, "a stage's last coefficient must not be zero (P:635-637)");
+        std::vector<uint64_t> nu(Nu.size() + ps, 0), du(Du.size() + ks, 0);
+        std::vector<double> nd(Nd.size() + ps, 0.0), dd(Dd.size() + ks, 0.0);
+        for (int j = 0; j <= ps; j++) {
+            const double v = ap[j];
+            if (dtype == PLR_INT32 && (v != std::floor(v) || std::fabs(v) >= 9.0e15))
+                return fail(PLR_ERR_SIGNATURE, "PLR_INT32 needs integer coefficients");
+            const uint64_t vu = (uint64_t)(int64_t)v;
+            const double vd = (double)(float)v;
+            for (size_t i = 0; i < Nu.size(); i++) { nu[i + j] += Nu[i] * vu; nd[i + j] += Nd[i] * vd; }
+        }
+        for (int j = 0; j <= ks; j++) {
+            const double v = j == 0 ? 1.0 : -bp[j - 1];
+            if (dtype == PLR_INT32 && (v != std::floor(v) || std::fabs(v) >= 9.0e15))
+                return fail(PLR_ERR_SIGNATURE, "PLR_INT32 needs integer coefficients");
+            const uint64_t vu = (uint64_t)(int64_t)v;
+            const double vd = j == 0 ? 1.0 : -(double)(float)bp[j - 1];
+            for (size_t i = 0; i < Du.size(); i++) { du[i + j] += Du[i] * vu; dd[i + j] += Dd[i] * vd; }
+        }
+        for (auto& e : nu) e &= 0xffffffffull;
+        for (auto& e : du) e &= 0xffffffffull;
+        Nu.swap(nu); Du.swap(du); Nd.swap(nd); Dd.swap(dd);
+        ap += ps + 1;
+        bp += ks;
+    }
+    const int P = (int)Nu.size() - 1, K = (int)Du.size() - 1;
+    if (K < 1) return fail(PLR_ERR_SIGNATURE, "the cascade has no feedback stage (k = 0, P:89-93)");
+    if (K > kMaxK || P > kMaxP) return fail(PLR_ERR_SIZE, "combined order exceeds PLR_MAX_K / PLR_MAX_P");
+    double ac[kMaxP + 1], bc[kMaxK];
+    for (int j = 0; j <= P; j++) ac[j] = dtype == PLR_INT32 ? (double)Nu[j] : Nd[j];
+    for (int j = 1; j <= K; j++)                       // b_j = -D_j
+        bc[j - 1] = dtype == PLR_INT32 ? (double)((0x100000000ull - Du[j]) & 0xffffffffull) : -Dd[j];
+    return plr_plan_create(out, ac, P, bc, K, dtype, n_max);
+}
+
+plr_status plr_plan_get_signature(const plr_plan* plan, double* a, double* b) {
+    if (plan == nullptr || a == nullptr || b == nullptr) return fail(PLR_ERR_INVALID_ARG, "null argument");
+    for (int j = 0; j <= plan->pt.p; j++) a[j] = plan->pt.dtype == PLR_INT32 ? (double)plan->pt.a_u[j] : plan->pt.a_d[j];
+    for (int j = 0; j < plan->pt.k; j++) b[j] = plan->pt.dtype == PLR_INT32 ? (double)plan->pt.b_u[j] : plan->pt.b_d[j];
     return PLR_OK;
 }
 
@@ -428,6 +537,8 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->const_sig = plan->sig_kernel ? plan->pt.sig_id : 0;
     info->tiles_per_unit = plan->pt.geo.G;
     info->kernel_kind = kernel_kind(plan->pt);
+    info->acc_bits = (plan->pt.dtype == PLR_FLOAT32 && plan->pt.acc64) ? 64 : 32;
+    info->cond_bound = plan->pt.dtype == PLR_FLOAT32 ? plan->pt.cond_bound : 0.0;
     return PLR_OK;
 }
 
@@ -611,12 +722,12 @@ plr_status plr_execute_sharded(plr_plan* plan, const void* x, void* y, size_t n,
         st = plr_reduce(plan, x, n, plan->d_send, stream);                          // reads n
     }
     if (st != PLR_OK) return st;
-    if (world > 1) {
+    if (comm != nullptr) {                      // the collective, also for a 1-rank communicator
         st = nccl_load();
         if (st != PLR_OK) return st;
         int r = g_nccl.allgather(plan->d_send, plan->d_recv, PLR_PAYLOAD_BYTES, /*ncclUint8*/ 1, comm, s);
         if (r != 0) return nccl_fail(r, "ncclAllGather");
-    } else {
+    } else {                                    // world == 1 without a communicator: loopback
         CUDA_TRY(cudaMemcpyAsync(plan->d_recv, plan->d_send, PLR_PAYLOAD_BYTES, cudaMemcpyDeviceToDevice, s), "copy");
     }
     st = plr_combine(plan, plan->d_recv, rank, world, plan->d_hist, stream);

@@ -94,7 +94,7 @@ PLR_HD constexpr Tables<T, A> const_tables(int sig, int X, int W, int G) {
         const CMat M = const_sig_companion(sig);
         const unsigned long long m = 32ull * W * X;
         t.alpha[0] = 1u;
-        for (int r = 0; r < k; r++) t.c[r] = const_sig_c(sig, r);
+        for (int r = 0; r < k; r++) t.c[r] = t.cT[r] = const_sig_c(sig, r);
         CMat Tu = M;                                   // T(u+1)
         for (int u = 0; u < kMaxX; u++) {
             for (int r = 0; r < kMaxK; r++) t.H[u][r] = (u < X) ? Tu.v[r] : 0u;

@@ -34,6 +34,18 @@ cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la) {
     return launch_scan_f32(pt.tf, la, pt.k, pt.p);
 }
 
+cudaError_t launch_small(const PlanTables& pt, const LaunchArgs& la) {
+    if (pt.dtype == PLR_INT32) return launch_small_i32(pt.tis, la, pt.k, pt.p);
+    if (pt.acc64) return launch_small_f64acc(pt.tds, la, pt.k, pt.p);
+    return launch_small_f32(pt.tfs, la, pt.k, pt.p);
+}
+
+cudaError_t small_occupancy(const PlanTables& pt, int* ctas_per_sm) {
+    LaunchArgs la{};
+    la.occupancy_out = ctas_per_sm;
+    return launch_small(pt, la);
+}
+
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm) {
     LaunchArgs la{};
     la.store = true;

@@ -41,6 +41,7 @@ template <typename T, typename A>
 struct Tables {
     T alpha[kMaxP + 1];                  // a0, a-1, ..., a-p       (FIR, data type)
     A c[kMaxK];                          // b-1, ..., b-k           (recurrence)
+    T cT[kMaxK];                         // b-1, ..., b-k in the data type (seeded phase B of the DECAY kernel)
     T H[kMaxX][kMaxK];                   // H[u][r] = h^(r+1)_u = T(u+1)[0][r], u < X
     A Twarp[5][kMaxK * kMaxK];           // T(X * 2^s)          lane scan
     A Tblk[4][kMaxK * kMaxK];            // T(32 X * 2^s)       warp-aggregate scan
@@ -88,6 +89,16 @@ struct PlanTables {
     Tables<float, double> td;            // fp32, fp64 accumulation
     Tables<uint32_t, uint32_t> ti1;      // ti / td with look-back units of one tile (Tpow = T(m 2^s))
     Tables<float, double> td1;
+    // small-n kernel (plr_kernels_small.cuh): its own tile geometry geo_s
+    Geometry geo_s;
+    Tables<uint32_t, uint32_t> tis;
+    Tables<float, float> tfs;
+    Tables<float, double> tds;
+    uint32_t lane_is[kMaxK * kMaxK * 32];
+    float lane_fs[kMaxK * kMaxK * 32];
+    double lane_ds[kMaxK * kMaxK * 32];
+    uint32_t dec_mask_s;                 // ScanParams::dec_mask of the small-n tables
+    int decay_s;                         // T(m_s) == 0 exactly (one-hop look-back)
     uint32_t lane_i[kMaxK * kMaxK * 32];
     float lane_f[kMaxK * kMaxK * 32];
     double lane_d[kMaxK * kMaxK * 32];
@@ -98,6 +109,10 @@ struct PlanTables {
     // (x_{-4..-1}, y_{-4..-1}) with zero input, i < fixup_len (fp32)
     float* fix_table;                    // host, fixup_len * kAug (owned)
 };
+
+// small-n kernel geometry: X = 15 elements per thread, W = 8 warps, m = 3840
+constexpr int kSmallX = 15;
+constexpr int kSmallW = 8;
 
 // planner (host, plr_planner.cpp)
 plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype dtype,

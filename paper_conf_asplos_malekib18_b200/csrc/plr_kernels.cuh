@@ -569,8 +569,13 @@ struct Layout {
 };
 
 // ------------------------------------------------------ the scan kernel ----
+// SEED: phase B evaluates the serial recurrence of P:206-214 over the
+// thread's X elements seeded with its true incoming state (the alternative
+// of SURVEY §8(a) a6) instead of correcting parked chunk values with the
+// factors h^(r)_u; the stage then holds the map outputs t (Eq. 2) between
+// the phases, or x itself when p = 0 (t = a0 x is recomputed).
 template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool DEC, bool STORE,
-          int MINB>
+          int MINB, bool SEED = false>
 __global__ void __launch_bounds__((W + 1 + NL) * 32, MINB)
 plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = Layout<T, A, K, X, W, S, D>;
@@ -798,9 +803,10 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             }
         }
         // a2: sequential local recurrence with zero state, in A
-        // chunk values are kept in the data type (phase B corrects them);
-        // only the last K live in the accumulation type.  The oldest term is
-        // added first so the newest value l_{u-1} is on the critical path once.
+        // chunk values are kept in the data type (phase B corrects them;
+        // SEED: the map outputs t are kept instead); only the last K live in
+        // the accumulation type.  The oldest term is added first so the
+        // newest value l_{u-1} is on the critical path once.
         T lf[X];
         A hist[K];                                              // hist[r-1] = l_{u-r}
 #pragma unroll
@@ -810,6 +816,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             T t = tb.alpha[0] * xv[P + u];
 #pragma unroll
             for (int q = 1; q <= P; q++) t = mad(tb.alpha[q], xv[P + u - q], t);
+            if constexpr (SEED) lf[u] = t;
             A acc = cvt<A, T>(t);
 #pragma unroll
             for (int r = K; r >= 1; r--)
@@ -817,7 +824,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #pragma unroll
             for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
             hist[0] = acc;
-            lf[u] = cvt<T, A>(acc);
+            if constexpr (!SEED) lf[u] = cvt<T, A>(acc);
         }
         A v[K];
 #pragma unroll
@@ -844,9 +851,13 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         }
         named_sync(1, NC);                                      // all x reads and wagg writes done
 
-        // keep the chunk values for phase B in place of x (data type)
+        // keep the chunk values (SEED: the map outputs t) for phase B in place
+        // of x (data type).  SEED with p = 0: the stage keeps x (t = a0 x is
+        // recomputed), except for the ragged tile the compute warps loaded
+        if (!SEED || P > 0 || ragged) {
 #pragma unroll
-        for (int u = 0; u < X; u++) st[kHalo + tid * X + u] = lf[u];
+            for (int u = 0; u < X; u++) st[kHalo + tid * X + u] = lf[u];
+        }
 
         // a4, DECAY with T(32X d) == 0 for d >= 1 (dec_mask bit 5 clear): the
         // exclusive warp prefix is the previous warp's aggregate and the tile
@@ -938,12 +949,27 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         for (int q = 0; q < K; q++) Sd[q] = cvt<T, A>(Sst[q]);
         T* base = st + kHalo + tid * X;
         T yv[X];
+        if constexpr (SEED) {
+            // a6: y_u = t_u + sum_r b-r y_{u-r}, seeded with Sd = (y_{-1}, ..., y_{-K})
+            const bool has_t = P > 0 || ragged;
 #pragma unroll
-        for (int u = 0; u < X; u++) {
-            T acc = base[u];
+            for (int u = 0; u < X; u++) {
+                T acc = has_t ? base[u] : tb.alpha[0] * base[u];
 #pragma unroll
-            for (int r = 0; r < K; r++) acc = mad(tb.H[u][r], Sd[r], acc);
-            yv[u] = acc;
+                for (int r = K; r >= 1; r--) acc = mad(tb.cT[r - 1], Sd[r - 1], acc);
+#pragma unroll
+                for (int r = K - 1; r >= 1; r--) Sd[r] = Sd[r - 1];
+                Sd[0] = acc;
+                yv[u] = acc;
+            }
+        } else {
+#pragma unroll
+            for (int u = 0; u < X; u++) {
+                T acc = base[u];
+#pragma unroll
+                for (int r = 0; r < K; r++) acc = mad(tb.H[u][r], Sd[r], acc);
+                yv[u] = acc;
+            }
         }
         if (!ragged) {
             if (STORE) {

@@ -30,11 +30,40 @@ struct LaunchArgs {
     int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel
 };
 
+// ScanParams of one launch from the plan's tables and the launch arguments
+template <typename T, typename A>
+inline ScanParams<T, A> make_params(const Tables<T, A>& tab, const LaunchArgs& la) {
+    ScanParams<T, A> prm;
+    prm.x = static_cast<const T*>(la.x);
+    prm.y = static_cast<T*>(la.y);
+    prm.n = la.n;
+    prm.ntiles = la.ntiles;
+    prm.ticket = la.ticket;
+    prm.status = la.status;
+    prm.status_mask = la.status_mask;
+    prm.decay = la.decay;
+    prm.dec_mask = la.dec_mask;
+    prm.x_hist = static_cast<const T*>(la.x_hist);
+    prm.y_hist = static_cast<const T*>(la.y_hist);
+    prm.y_tail = static_cast<T*>(la.y_tail);
+    prm.lane_T = static_cast<const A*>(la.lane_T);
+    prm.stats = la.stats;
+    prm.tab = tab;
+    return prm;
+}
+
 // Tile geometry of the DECAY / generic kernel configs.
 // (fp64-accumulation DECAY plans have their own config)
 Geometry class_geometry(bool decay, int k, bool acc64 = false);
 
 cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
+// the small-n kernel (plr_kernels_small.cuh): one CTA per tile of the plan's
+// geo_s, grid = ntiles (la.grid ignored); la.y == nullptr: reduce-only
+cudaError_t launch_small(const PlanTables& pt, const LaunchArgs& la);
+cudaError_t small_occupancy(const PlanTables& pt, int* ctas_per_sm);
+cudaError_t launch_small_i32(const Tables<uint32_t, uint32_t>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_small_f32(const Tables<float, float>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_small_f64acc(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm);
 
 // per-(data, accumulation) type entry points (plr_scan_*.cu)

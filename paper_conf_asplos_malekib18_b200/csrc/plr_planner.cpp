@@ -182,6 +182,8 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
     PlanTables& pt = *out;
     std::memset(&pt, 0, sizeof(pt));
     pt.p = p; pt.k = k; pt.dtype = dtype; pt.geo = geo;
+    pt.geo_s = Geometry{kSmallX, kSmallW, 1, 1};
+    pt.dec_mask_s = 0x3fu;
     pt.decay_len = -1; pt.fixup_len = 0;
     pt.dec_mask = 0x3fu;
     pt.fix_table = nullptr;
@@ -191,7 +193,7 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         for (int j = 0; j <= p; j++) pt.a_u[j] = (uint32_t)(int64_t)(a[j] < 0 ? a[j] : std::fmod(a[j], 4294967296.0));
         for (int j = 0; j < k; j++) c[j] = pt.b_u[j] = (uint32_t)(int64_t)(b[j] < 0 ? b[j] : std::fmod(b[j], 4294967296.0));
         for (int j = 0; j <= kMaxP; j++) pt.ti.alpha[j] = j <= p ? pt.a_u[j] : 0u;
-        for (int j = 0; j < kMaxK; j++) pt.ti.c[j] = j < k ? c[j] : 0u;
+        for (int j = 0; j < kMaxK; j++) pt.ti.c[j] = pt.ti.cT[j] = j < k ? c[j] : 0u;
         Mat<uint32_t> M = companion<uint32_t>(c, k);
         auto id = [](uint32_t v) { return v; };
         fill_tables(M, k, geo, &pt.ti, pt.lane_i, id, id);
@@ -202,6 +204,8 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
             pt.ti1 = pt.ti;                    // coefficients (alpha, c); the matrices are refilled
             fill_tables(M, k, g1, &pt.ti1, lane_tmp, id, id);
         }
+        pt.tis = pt.ti;                        // small-n kernel tables (own geometry, units of one tile)
+        fill_tables(M, k, pt.geo_s, &pt.tis, pt.lane_is, id, id);
         // class: all factors 1 -> ONES; single unit feedback
         // coefficient -> PERM (0/1 repeating factors); otherwise POLY
         int nnz = 0, ones = 0;
@@ -228,6 +232,7 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         for (int j = 0; j <= kMaxP; j++) pt.tf.alpha[j] = pt.td.alpha[j] = j <= p ? (float)al[j] : 0.0f;
         for (int j = 0; j < kMaxK; j++) pt.tf.c[j] = j < k ? (float)c[j] : 0.0f;
         for (int j = 0; j < kMaxK; j++) pt.td.c[j] = j < k ? c[j] : 0.0;
+        for (int j = 0; j < kMaxK; j++) pt.tf.cT[j] = pt.td.cT[j] = j < k ? (float)c[j] : 0.0f;
         Mat<double> M = companion<double>(c, k);
         auto f32 = [](double v) { return ftz(v); };
         // fp64 accumulation keeps denormal-range values that fp32 would flush;
@@ -242,6 +247,10 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
             pt.td1 = pt.td;                    // coefficients (alpha, c); the matrices are refilled
             fill_tables(M, k, g1, &pt.td1, lane_tmp, f32, f64);
         }
+        pt.tfs = pt.tf;                        // small-n kernel tables (own geometry, units of one tile)
+        pt.tds = pt.td;
+        fill_tables(M, k, pt.geo_s, &pt.tfs, pt.lane_fs, f32, f32);
+        fill_tables(M, k, pt.geo_s, &pt.tds, pt.lane_ds, f32, f64);
         // DECAY: the fp32 impulse response g of (1: c) becomes
         // exactly 0 and stays 0.  g_0 = 1, g_u = sum_j c_j g_{u-j}.
         const int64_t cap = 1 << 16;
@@ -259,21 +268,37 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         pt.decay_flag = (decays && tm_zero) ? 1 : 0;
         pt.cls = decays ? PLR_CLASS_DECAY : PLR_CLASS_FLOAT;
         // Accumulation precision (reading R16).  The zero-state
-        // chunk values l_u and the carries reach ~sum|a| * sum|g| while the
-        // outputs stay small, and their rounding errors are amplified by the
-        // correction factors again (~sum|g|): a-priori bound
-        // eps32 * sum|a| * (sum|g|)^2.  Above 1e-3 (10x the 1e-4 tolerance)
-        // accumulate the recurrence and every carry in fp64 (B200 fp64 runs at
-        // half the fp32 rate); data, FIR and the final correction stay fp32.
+        // chunk values l_u and the carries reach ~sum|a| * sum|g| times the
+        // input scale, and their rounding errors are amplified by the
+        // transfer matrices again (~sum|g|): a-priori bound
+        // eps32 * sum|a| * (sum|g|)^2 relative to the input scale.  The
+        // tolerance is relative to the OUTPUT (1e-4 max(1,|y|)), so the bound
+        // is divided by the gain the filter leaves an input at the Nyquist
+        // frequency -- the worked example's (-1)^i (i+3) pattern, the
+        // input a low-pass filter attenuates most: |H(-1)| = |A(-1)| / |B(-1)|
+        // (capped at 1).  Above 1e-3 (10x the tolerance) the chunk recurrence
+        // and every carry accumulate in fp64 (B200 fp64 runs at half the fp32
+        // rate); data, the map and phase B stay fp32.
         double sa = 0.0, sg = 0.0;
         for (int j = 0; j <= p; j++) sa += std::fabs(al[j]);
         for (int64_t u = 0; u < cap; u++) sg += std::fabs(g[u]);
-        pt.cond_bound = std::ldexp(1.0, -24) * sa * sg * sg;
+        double an = 0.0, bn = 1.0;                       // A(-1), B(-1) = 1 - sum_j c_j (-1)^j
+        for (int j = 0; j <= p; j++) an += (j & 1) ? -al[j] : al[j];
+        for (int j = 1; j <= k; j++) bn -= (j & 1) ? -c[j - 1] : c[j - 1];
+        const double nyq = bn != 0.0 ? std::fabs(an / bn) : 1.0;
+        pt.cond_bound = std::ldexp(1.0, -24) * sa * sg * sg / std::fmin(1.0, nyq);
         pt.acc64 = (!decays || !(pt.cond_bound <= 1e-3)) ? 1 : 0;
         if (!pt.decay_flag) pt.acc64 = 1;      // multi-tile look-back kernels exist in fp64 accumulation only
         pt.dec_mask = 0x3fu;
         if (pt.decay_flag)                     // DECAY hierarchy: skip the negligible transfer matrices
             pt.dec_mask = pt.acc64 ? decay_mask(&pt.td, pt.lane_d, k, geo) : decay_mask(&pt.tf, pt.lane_f, k, geo);
+        bool tms_zero = true;
+        for (int e = 0; e < kMaxK * kMaxK; e++) tms_zero = tms_zero && pt.tfs.Tm[e] == 0.0f && pt.tds.Tm[e] == 0.0;
+        pt.decay_s = (decays && tms_zero) ? 1 : 0;
+        pt.dec_mask_s = 0x3fu;
+        if (pt.decay_s)
+            pt.dec_mask_s = pt.acc64 ? decay_mask(&pt.tds, pt.lane_ds, k, pt.geo_s)
+                                     : decay_mask(&pt.tfs, pt.lane_fs, k, pt.geo_s);
         if (decays) {
             pt.decay_len = last;
             // free response of the augmented state (x_{-4..-1}, y_{-4..-1})

@@ -111,13 +111,20 @@ constexpr int gen_kind(int k) { return k == 1 ? PLR_K1_KIND : PLR_GEN_KIND; }
 // W compute warps (tile m = 32 W X); MINB: CTAs per SM the registers must allow
 // U1_: look-back units of one tile (the small-n launches, plr_api.cu), else
 // PLR_RR_G / PLR_TM_G tiles per unit
-template <int S_, int D_, int NL_, int X_, int W_, int MINB_, bool DEC_, bool U1_ = false>
+// SEED_: phase B runs the seeded serial recurrence (plr_scan_kernel SEED)
+template <int S_, int D_, int NL_, int X_, int W_, int MINB_, bool DEC_, bool U1_ = false, bool SEED_ = false>
 struct Cfg {
     static constexpr int S = S_, D = D_, NL = NL_, X = X_, W = W_, MINB = MINB_;
-    static constexpr bool DEC = DEC_, U1 = U1_;
+    static constexpr bool DEC = DEC_, U1 = U1_, SEED = SEED_;
 };
-using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true>;
-using CfgDec64 = Cfg<PLR_DEC64_S, PLR_DEC64_D, PLR_DEC64_NL, PLR_DEC64_X, PLR_DEC64_W, PLR_DEC64_MINB, true>;
+// DECAY kernels: phase B seeded with the true carry (PLR_DEC_SEED=0: the
+// correction y = l + sum_r S_r h^(r)_u, kept for comparison builds)
+#ifndef PLR_DEC_SEED
+#define PLR_DEC_SEED 1
+#endif
+using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true, false, PLR_DEC_SEED>;
+using CfgDec64 = Cfg<PLR_DEC64_S, PLR_DEC64_D, PLR_DEC64_NL, PLR_DEC64_X, PLR_DEC64_W, PLR_DEC64_MINB, true, false,
+                     PLR_DEC_SEED>;
 using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false>;
 using CfgGen1 = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false, true>;
 
@@ -151,7 +158,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
         smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
         threads = (TC::W + 1 + TC::NL) * 32;
     } else {
-        kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB>;
+        kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB, C::SEED>;
         smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
         threads = (C::W + 1 + C::NL) * 32;
     }
@@ -171,22 +178,7 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
         if (tmem && *la.occupancy_out > 1) *la.occupancy_out = 1;   // 512 TMEM columns per CTA
         return e;
     }
-    ScanParams<T, A> prm;
-    prm.x = static_cast<const T*>(la.x);
-    prm.y = static_cast<T*>(la.y);
-    prm.n = la.n;
-    prm.ntiles = la.ntiles;
-    prm.ticket = la.ticket;
-    prm.status = la.status;
-    prm.status_mask = la.status_mask;
-    prm.decay = la.decay;
-    prm.dec_mask = la.dec_mask;
-    prm.x_hist = static_cast<const T*>(la.x_hist);
-    prm.y_hist = static_cast<const T*>(la.y_hist);
-    prm.y_tail = static_cast<T*>(la.y_tail);
-    prm.lane_T = static_cast<const A*>(la.lane_T);
-    prm.stats = la.stats;
-    prm.tab = tab;
+    const ScanParams<T, A> prm = make_params(tab, la);
     kern<<<la.grid, threads, smem, la.stream>>>(prm);
     return cudaGetLastError();
 }

@@ -28,7 +28,7 @@ def test_exports_every_declared_symbol():
     for s in syms:
         assert hasattr(plr.lib, s), s
     assert set(syms) == set(plr.binding.EXPORTED)
-    assert plr.abi_version() == 2
+    assert plr.abi_version() == 3
 
 
 @pytest.mark.parametrize("a,b,dtype,code", [
@@ -55,6 +55,23 @@ def test_classes():
     for nm in ("lp1", "lp2", "lp3", "hp1", "hp2", "hp3"):
         assert cls[nm] == "DECAY"
     assert plr.Plan((1.0,), (1.0,), "float32", n_max=0).info["cls"] == "FLOAT"
+
+
+def test_precision_rule_r16():
+    """DESIGN.md reading R16: fp64 accumulation when the a-priori fp32 bound
+    eps32 sum|a| (sum|g|)^2 / min(1, |H(-1)|) exceeds 1e-3.  Closed forms for
+    (a0: c) with the pole 0.8 of multiplicity s (LP_s, Table 1):
+    sum|g| = 0.2^-s and |H(-1)| = a0 / 1.8^s."""
+    eps = 2.0 ** -24
+    for name, s in (("lp1", 1), ("lp2", 2), ("lp3", 3)):
+        sig = workloads.BY_NAME[name]
+        info = plr.Plan(sig.a, sig.b, sig.dtype, n_max=0).info
+        a0 = float(np.float32(sig.a[0]))
+        bound = eps * a0 * (0.2 ** -s) ** 2 / min(1.0, a0 / 1.8 ** s)
+        assert info["cond_bound"] == pytest.approx(bound, rel=1e-4), name
+    acc = {s.name: plr.Plan(s.a, s.b, s.dtype, n_max=0).info["acc_bits"] for s in workloads.TABLE1}
+    assert acc == {"prefix": 32, "tuple2": 32, "tuple3": 32, "order2": 32, "order3": 32,
+                   "lp1": 32, "lp2": 32, "lp3": 64, "hp1": 32, "hp2": 32, "hp3": 64}
 
 
 def test_decay_length_matches_ftz_threshold():
@@ -134,3 +151,33 @@ def test_combine_host_matches_oracle(sig):
             assert np.array_equal(h[4:], ex_y.astype(np.int32))
         else:
             np.testing.assert_allclose(h[4:], ex_y, rtol=1e-5, atol=1e-5)
+
+
+# ------------------------------------------------------------ cascade ------
+def test_cascade_combines_polynomials():
+    """plr_plan_create_cascade multiplies the stages' z-transforms:
+    three prefix sums -> (1: 3, -3, 1); a FIR stage with a tuple
+    sum and a 2nd-order sum -> (3, -1 : 2, 0, -2, 1) in Z/2^32; three 1-stage
+    high-pass filters -> the untruncated 3-stage high-pass row (reading R4)."""
+    pl = plr.Plan.cascade([((1,), (1,))] * 3, "int32", n_max=0)
+    assert (pl.p, pl.k) == (0, 3)
+    assert pl.a == (1.0,) and pl.b == (3.0, float(2 ** 32 - 3), 1.0)
+    pl = plr.Plan.cascade([((3, -1), (0, 1)), ((1,), (2, -1))], "int32", n_max=0)
+    assert pl.a == (3.0, float(2 ** 32 - 1)) and pl.b == (2.0, 0.0, float(2 ** 32 - 2), 1.0)
+    pl = plr.Plan.cascade([((0.9, -0.9), (0.8,))] * 3, "float32", n_max=0)
+    hp3 = workloads.BY_NAME["hp3"]
+    np.testing.assert_allclose(pl.a, hp3.a, rtol=1e-6)
+    np.testing.assert_allclose(pl.b, hp3.b, rtol=1e-6)
+    assert pl.info["cls"] == "DECAY"
+
+
+@pytest.mark.parametrize("stages,code", [
+    ([((1,), ())], 2),                                   # no feedback stage at all (P:89-93)
+    ([((1,), (1, 0))], 2),                               # a stage's trailing zero (P:635-637)
+    ([((1,), (1,))] * 5, 4),                             # combined k = 5 > PLR_MAX_K
+    ([((1, 1), (1,))] * 4, 4),                           # combined p = 4 > PLR_MAX_P
+])
+def test_cascade_validation(stages, code):
+    with pytest.raises(plr.PLRError) as e:
+        plr.Plan.cascade(stages, "int32", n_max=0)
+    assert e.value.status == code

@@ -45,9 +45,24 @@ def sizes_for(m):
             (1 << 16) + 3, (1 << 20) + 12345]
 
 
+# "auto": the size-dependent kernel choice (the small-n kernel up to
+# PLR_SMALL_MAX elements); "big": PLR_SMALL_MAX=0, the persistent kernels at
+# every size
+PATHS = {"auto": None, "big": "0"}
+
+
+def use_path(monkeypatch, path):
+    if PATHS[path] is None:
+        monkeypatch.delenv("PLR_SMALL_MAX", raising=False)
+    else:
+        monkeypatch.setenv("PLR_SMALL_MAX", PATHS[path])
+
+
 @pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
-def test_parity_sizes(cuda_plr, sig):
+@pytest.mark.parametrize("path", sorted(PATHS))
+def test_parity_sizes(cuda_plr, sig, path, monkeypatch):
     import torch
+    use_path(monkeypatch, path)
     m = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 10).info["tile_elems"]
     SIZES = sizes_for(m)
     x_all = workloads.host_input(max(SIZES), sig.dtype, workloads.seed_for(1))
@@ -60,8 +75,10 @@ def test_parity_sizes(cuda_plr, sig):
 
 @pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
 @pytest.mark.parametrize("kind", ["ones", "impulse", "alternating", "extremes"])
-def test_parity_structured(cuda_plr, sig, kind):
+@pytest.mark.parametrize("path", sorted(PATHS))
+def test_parity_structured(cuda_plr, sig, kind, path, monkeypatch):
     import torch
+    use_path(monkeypatch, path)
     n = 7 * M + 123
     x = workloads.structured_input(kind, n, sig.dtype)
     y = run(cuda_plr, torch, sig, x)
@@ -90,10 +107,12 @@ def test_closed_forms_on_gpu(cuda_plr):
 
 
 @pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
-def test_repeated_launches_epochs(cuda_plr, sig):
+def test_repeated_launches_epochs(cuda_plr, sig, monkeypatch):
     """One plan, many launches with varying n: epoch-tagged status words and
-    the ticket base must never mix launches."""
+    the ticket base must never mix launches -- also across the small-n and
+    the persistent kernels, which share the plan's launch state."""
     import torch
+    monkeypatch.setenv("PLR_SMALL_MAX", str(60 * M))
     plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=200 * M)
     rng = np.random.default_rng(5)
     for t in range(12):
@@ -104,7 +123,7 @@ def test_repeated_launches_epochs(cuda_plr, sig):
 
 
 @pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
-@pytest.mark.parametrize("n", [5000, 3 * M + 7, (1 << 20) + 12345])
+@pytest.mark.parametrize("n", [5000, 3 * M + 7, (1 << 20) + 12345, (1 << 22) + 4321])
 def test_cuda_graph_replay(cuda_plr, sig, n):
     """plr_execute captured in a CUDA graph: the ticket base and the epoch
     live on the device (launch_state_advance), so every replay, and eager
@@ -313,6 +332,7 @@ def test_ablation_modes_parity(cuda_plr, sig, mode, monkeypatch):
     import torch
     var, val = ABLATIONS[mode]
     monkeypatch.setenv(var, val)
+    monkeypatch.setenv("PLR_SMALL_MAX", "0")          # the persistent kernels the ablation times
     probe = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 10)
     m = probe.info["tile_elems"]
     if mode == "generic":
@@ -359,4 +379,22 @@ def test_decay_bitwise_repeatable(cuda_plr, sig):
         torch.cuda.synchronize()
         assert np.array_equal(y, first), "%s: run %d differs bitwise in %d elements" % (
             sig.name, t, int(np.count_nonzero(y != first)))
+    plan.close()
+
+
+# ------------------------------------------------------------ small n ------
+@pytest.mark.parametrize("sig", workloads.TABLE1, ids=lambda s: s.name)
+def test_small_n_sweep_points(cuda_plr, sig, monkeypatch):
+    """every size of the sweep 2^10 .. 2^22
+    plus ragged neighbours, through the size-dependent kernel choice, and
+    the small-n kernel forced beyond its default range (2^22 + 777)."""
+    import torch
+    sizes = [1 << e for e in range(10, 23)] + [(1 << e) + 5 for e in (10, 16, 21)] + [(1 << 22) + 777]
+    x_all = workloads.host_input(max(sizes), sig.dtype, workloads.seed_for(11))
+    monkeypatch.setenv("PLR_SMALL_MAX", str(max(sizes)))
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=max(sizes))
+    for n in sizes:
+        x = x_all[:n].copy()
+        y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+        check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s n=%d" % (sig.name, n))
     plan.close()

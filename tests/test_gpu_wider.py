@@ -35,10 +35,16 @@ def check(y, ref, sig, what):
 
 
 @pytest.mark.parametrize("sig", WIDER, ids=lambda s: s.name)
-@pytest.mark.parametrize("waves", ["4", "0"])
+@pytest.mark.parametrize("waves", ["4", "0", "small"])
 def test_wider_signatures(cuda_plr, sig, waves, monkeypatch):
+    """waves "4" / "0": the persistent kernels (PLR_SMALL_MAX=0) with look-back
+    units of one tile / of G tiles; "small": the small-n kernel at every size."""
     import torch
-    monkeypatch.setenv("PLR_UNIT1_WAVES", waves)
+    if waves == "small":
+        monkeypatch.setenv("PLR_SMALL_MAX", str(1 << 22))
+    else:
+        monkeypatch.setenv("PLR_SMALL_MAX", "0")
+        monkeypatch.setenv("PLR_UNIT1_WAVES", waves)
     m = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 10).info["tile_elems"]
     sizes = [1, 5, m - 1, m + 1, 7 * m + 3, 33 * m + 5, (1 << 20) + 12345]
     x_all = workloads.host_input(max(sizes), sig.dtype, workloads.seed_for(7))

@@ -60,5 +60,5 @@ for sig in workloads.TABLE1:
     wa, _ = rel(ya, oracle.recurrence(xa, sig.a, sig.b, sig.dtype))
     pa.close()
     print("| %s | %s | %s | %.3g | %d | %.3g | 1e-4 |" % (
-        sig.name, info.get("kernel_kind"), info.get("acc", "?"), w, i, wa), flush=True)
+        sig.name, info.get("kernel_kind"), info.get("acc_bits", "?"), w, i, wa), flush=True)
     sys.stderr.write("%s %.1fs\n" % (sig.name, time.time() - t0))
