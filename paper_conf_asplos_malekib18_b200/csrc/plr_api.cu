@@ -48,6 +48,8 @@ struct plr_plan {
     void* d_lane = nullptr;
     void* d_lane_s = nullptr;           // lane table T(X_s l) of the small-n kernel
     size_t small_max = 0;               // n <= small_max: the small-n kernel (plr_kernels_small.cuh)
+    int reduce_ctas = 0;                // CTAs per SM of the reduce-only kernel (0: not available)
+    unsigned long long* d_rd = nullptr; // its per-CTA records (kStatusMaxBytes each)
     float* d_fix = nullptr;
     bool dirty = false;
     bool sig_kernel = false;            // launch the compile-time signature kernel (pt.sig_id)
@@ -341,6 +343,7 @@ plr_status plr_plan_destroy(plr_plan* plan) {
     cudaFree(plan->d_status);
     cudaFree(plan->d_lane);
     cudaFree(plan->d_lane_s);
+    cudaFree(plan->d_rd);
     cudaFree(plan->d_fix);
     cudaFree(plan->d_send);
     cudaFree(plan->d_recv);
@@ -416,6 +419,13 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     if (plan->ctas_per_sm < 1) { plr_plan_destroy(plan); return fail(PLR_ERR_CUDA, "kernel does not fit on an SM"); }
     int small_ctas = 0;
     if ((e = small_occupancy(plan->pt, &small_ctas)) != cudaSuccess) return bail(e, "occupancy (small-n)");
+    if (plan->pt.dtype == PLR_INT32 || plan->pt.acc64) {     // non-DECAY capable: the reduce-only kernel
+        if ((e = reduce_occupancy(plan->pt, &plan->reduce_ctas)) != cudaSuccess) return bail(e, "occupancy (reduce)");
+        if (plan->reduce_ctas > 0) {
+            const size_t rb = (size_t)plan->num_sms * plan->reduce_ctas * kStatusMaxBytes;
+            if ((e = cudaMalloc(&plan->d_rd, rb)) != cudaSuccess) return bail(e, "alloc reduce records");
+        }
+    }
     plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default()) : 0;
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
@@ -581,8 +591,37 @@ plr_status plr_reduce(plr_plan* plan, const void* x, size_t n, void* payload, vo
     CUDA_TRY(cudaMemsetAsync(payload, 0, PLR_PAYLOAD_BYTES, s), "payload memset");
     if (n > 0) {
         uint32_t* y_tail = reinterpret_cast<uint32_t*>((unsigned char*)payload + 24) + (4 - plan->pt.k);
-        st = launch(plan, x, nullptr, n, nullptr, nullptr, y_tail, false, s);
-        if (st != PLR_OK) return st;
+        if (n > plan->n_max) return fail(PLR_ERR_SIZE, "n exceeds the plan's n_max");
+        if (n > plan->small_max && plan->d_rd != nullptr && std::getenv("PLR_NO_REDUCE_KERNEL") == nullptr) {
+            // contiguous-range streaming fold, no look-back (plr_kernels_reduce.cuh)
+            if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
+                CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, s), "status reset");
+                CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, kTicketBytes, s), "ticket reset");
+                plan->epoch = 0;
+                plan->dirty = false;
+            }
+            plan->epoch++;
+            const uint64_t m = (uint64_t)kRedX * kRedW * 32;
+            LaunchArgs la;
+            la.x = x; la.y = nullptr; la.n = n; la.ntiles = (n + m - 1) / m;
+            la.ticket = plan->d_ticket;
+            la.status = plan->d_rd;
+            la.status_mask = 0;
+            la.decay = 0;
+            la.x_hist = nullptr; la.y_hist = nullptr; la.y_tail = y_tail;
+            la.lane_T = nullptr;
+            la.grid = (int)std::min<uint64_t>(la.ntiles, (uint64_t)plan->num_sms * plan->reduce_ctas);
+            la.store = false;
+            la.stream = s;
+            cudaError_t e = launch_reduce(plan->pt, la);
+            if (e != cudaSuccess) {
+                plan->dirty = true;
+                return cuda_fail(e, "reduce kernel launch");
+            }
+        } else {
+            st = launch(plan, x, nullptr, n, nullptr, nullptr, y_tail, false, s);
+            if (st != PLR_OK) return st;
+        }
     }
     payload_kernel<<<1, 32, 0, s>>>((const uint32_t*)x, nullptr, n, (unsigned char*)payload, 0);
     CUDA_TRY(cudaGetLastError(), "payload kernel");

@@ -40,6 +40,18 @@ cudaError_t launch_small(const PlanTables& pt, const LaunchArgs& la) {
     return launch_small_f32(pt.tfs, la, pt.k, pt.p);
 }
 
+cudaError_t launch_reduce(const PlanTables& pt, const LaunchArgs& la) {
+    if (pt.dtype == PLR_INT32) return launch_reduce_i32(pt.tr, la, pt.k, pt.p);
+    if (pt.acc64) return launch_reduce_f64acc(pt.trd, la, pt.k, pt.p);
+    return cudaErrorInvalidValue;                       // fp32-accumulation plans are DECAY: no reduce pass
+}
+
+cudaError_t reduce_occupancy(const PlanTables& pt, int* ctas_per_sm) {
+    LaunchArgs la{};
+    la.occupancy_out = ctas_per_sm;
+    return launch_reduce(pt, la);
+}
+
 cudaError_t small_occupancy(const PlanTables& pt, int* ctas_per_sm) {
     LaunchArgs la{};
     la.occupancy_out = ctas_per_sm;

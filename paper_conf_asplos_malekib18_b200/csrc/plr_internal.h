@@ -98,6 +98,8 @@ struct PlanTables {
     float lane_fs[kMaxK * kMaxK * 32];
     double lane_ds[kMaxK * kMaxK * 32];
     uint32_t dec_mask_s;                 // ScanParams::dec_mask of the small-n tables
+    Tables<uint32_t, uint32_t> tr;       // reduce-only kernel tables (its own tile geometry)
+    Tables<float, double> trd;
     int decay_s;                         // T(m_s) == 0 exactly (one-hop look-back)
     uint32_t lane_i[kMaxK * kMaxK * 32];
     float lane_f[kMaxK * kMaxK * 32];
@@ -113,6 +115,11 @@ struct PlanTables {
 // small-n kernel geometry: X = 15 elements per thread, W = 8 warps, m = 3840
 constexpr int kSmallX = 15;
 constexpr int kSmallW = 8;
+// reduce-only kernel geometry (plr_kernels_reduce.cuh): X = 31, W = 8
+// (tile 7936), 3-stage TMA ring, 2 CTAs per SM
+constexpr int kRedX = 31;
+constexpr int kRedW = 8;
+constexpr int kRedS = 3;
 
 // planner (host, plr_planner.cpp)
 plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype dtype,

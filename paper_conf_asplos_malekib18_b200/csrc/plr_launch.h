@@ -61,6 +61,13 @@ cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
 // geo_s, grid = ntiles (la.grid ignored); la.y == nullptr: reduce-only
 cudaError_t launch_small(const PlanTables& pt, const LaunchArgs& la);
 cudaError_t small_occupancy(const PlanTables& pt, int* ctas_per_sm);
+// the reduce-only kernel (plr_kernels_reduce.cuh): la.status = per-CTA record
+// scratch (kStatusMaxBytes each), la.grid CTAs over contiguous tile ranges of
+// kRedX * kRedW * 32 elements, la.y_tail = the K end-state outputs
+cudaError_t launch_reduce(const PlanTables& pt, const LaunchArgs& la);
+cudaError_t reduce_occupancy(const PlanTables& pt, int* ctas_per_sm);
+cudaError_t launch_reduce_i32(const Tables<uint32_t, uint32_t>& tab, const LaunchArgs& la, int k, int p);
+cudaError_t launch_reduce_f64acc(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t launch_small_i32(const Tables<uint32_t, uint32_t>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t launch_small_f32(const Tables<float, float>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t launch_small_f64acc(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);

@@ -206,6 +206,11 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         }
         pt.tis = pt.ti;                        // small-n kernel tables (own geometry, units of one tile)
         fill_tables(M, k, pt.geo_s, &pt.tis, pt.lane_is, id, id);
+        {
+            uint32_t lane_tmp[kMaxK * kMaxK * 32];
+            pt.tr = pt.ti;                     // reduce-only kernel tables
+            fill_tables(M, k, Geometry{kRedX, kRedW, kRedS, 1}, &pt.tr, lane_tmp, id, id);
+        }
         // class: all factors 1 -> ONES; single unit feedback
         // coefficient -> PERM (0/1 repeating factors); otherwise POLY
         int nnz = 0, ones = 0;
@@ -251,6 +256,11 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         pt.tds = pt.td;
         fill_tables(M, k, pt.geo_s, &pt.tfs, pt.lane_fs, f32, f32);
         fill_tables(M, k, pt.geo_s, &pt.tds, pt.lane_ds, f32, f64);
+        {
+            double lane_tmp[kMaxK * kMaxK * 32];
+            pt.trd = pt.td;                    // reduce-only kernel tables
+            fill_tables(M, k, Geometry{kRedX, kRedW, kRedS, 1}, &pt.trd, lane_tmp, f32, f64);
+        }
         // DECAY: the fp32 impulse response g of (1: c) becomes
         // exactly 0 and stays 0.  g_0 = 1, g_u = sum_j c_j g_{u-j}.
         const int64_t cap = 1 << 16;

@@ -398,3 +398,30 @@ def test_small_n_sweep_points(cuda_plr, sig, monkeypatch):
         y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
         check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s n=%d" % (sig.name, n))
     plan.close()
+
+
+# ------------------------------------------------------------ reduce-only --
+@pytest.mark.parametrize("name", ["prefix", "tuple3", "order2", "order3", "fir_order2", "fsum"])
+@pytest.mark.parametrize("n", [(1 << 22) + 1, 7936 * 1000, (1 << 24) + 12345, 148 * 2 * 7936 * 3 - 4])
+def test_reduce_kernel_end_state(cuda_plr, name, n):
+    """plr_reduce beyond the small-n range runs the contiguous-range
+    streaming fold (plr_kernels_reduce.cuh): its payload's last k outputs
+    equal the oracle's y_{n-k} .. y_{n-1} of the zero-history segment (int32
+    bit-exact; float within the bar), incl. ragged ends and one tile per CTA
+    short of a full wave."""
+    import torch
+    sigs = {s.name: s for s in workloads.TABLE1}
+    sigs["fir_order2"] = workloads.Signature("fir_order2", (3, -1, 2, 5), (2, -1), "int32", "", "")
+    sigs["fsum"] = workloads.Signature("fsum", (1.0,), (1.0,), "float32", "", "")
+    sig = sigs[name]
+    x = workloads.host_input(n, sig.dtype, workloads.seed_for(14))
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    pl = plan.reduce(torch.from_numpy(x).cuda()).cpu().numpy()
+    ref = oracle.recurrence(x, sig.a, sig.b, sig.dtype)
+    assert int(pl[:8].view(np.uint64)[0]) == n
+    npdt = np.int32 if sig.dtype == "int32" else np.float32
+    got = pl[24:40].view(npdt)[4 - sig.k:]
+    xt = pl[8:24].view(npdt)
+    assert np.array_equal(xt, x[n - 4:])
+    check(got.astype(np.float64) if sig.dtype == "float32" else got, ref[n - sig.k:], sig.dtype, "%s n=%d" % (name, n))
+    plan.close()
