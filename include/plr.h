@@ -165,6 +165,23 @@ plr_status plr_plan_debug_stats(plr_plan* plan, uint64_t* out /* 16 */, int rese
  * x, y: device pointers of the plan's dtype. */
 plr_status plr_execute(plr_plan* plan, const void* x, void* y, size_t n, void* stream);
 
+/* The anticausal recurrence over x[0..n):
+ *     y_i = a0 x_i + a-1 x_{i+1} + ... + a-p x_{i+p} + b-1 y_{i+1} + ... + b-k y_{i+k},
+ * with x_j = y_j = 0 for j >= n -- Eq. (1) run from the end of the data to its
+ * start, the backward half of the causal/anticausal filter pairs of P:809-811
+ * and P:866-868.  Same layout, alignment and aliasing rules as plr_execute
+ * (x == y allowed when p == 0).  One pass: tiles are processed from the end
+ * with the same hierarchy and look-back. */
+plr_status plr_execute_reverse(plr_plan* plan, const void* x, void* y, size_t n, void* stream);
+
+/* Forward-backward (zero-phase) filtering: y = reverse(forward(x)), i.e. the
+ * causal recurrence then the anticausal one (plr_execute_reverse) on its
+ * output, two passes.  tmp (device, n elements of the dtype) holds the
+ * intermediate; it may be NULL when p == 0 (the backward pass then runs in
+ * place in y).  The intermediate is rounded to the dtype. */
+plr_status plr_execute_bidirectional(plr_plan* plan, const void* x, void* y, size_t n, void* tmp,
+                                     void* stream);
+
 /* Same, continuing a sequence: x_hist points at the p inputs before x[0]
  * (x_{-p}..x_{-1}, index order) and y_hist at the k outputs before y[0]
  * (y_{-k}..y_{-1}).  Either may be NULL (zeros).  For a long array split in

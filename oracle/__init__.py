@@ -56,6 +56,8 @@ def _load():
             lib.oracle_eq1_i32.argtypes = [P, P, I64, P, I, P, I, P, P]
             lib.oracle_eq1_f64.argtypes = [P, P, I64, P, I, P, I, P, P]
             lib.oracle_eq1_f64_dd.argtypes = [P, P, I64, P, I, P, I]
+            lib.oracle_rev_i32.argtypes = [P, P, I64, P, I, P, I]
+            lib.oracle_rev_f64.argtypes = [P, P, I64, P, I, P, I]
             lib.oracle_factor_lists_i32.argtypes = [P, I, I64, P]
             lib.oracle_factor_lists_f64.argtypes = [P, I, I64, P]
             lib.oracle_phase1_i32.argtypes = [P, I64, P, I, I64, P, I64, P]
@@ -144,6 +146,33 @@ def cascade(x, stages, dtype: str) -> np.ndarray:
             y = out
         return y
     raise ValueError(dtype)
+
+
+def anticausal(x, a, b, dtype: str) -> np.ndarray:
+    """The anticausal recurrence (Eq. (1) run from the end, zero beyond it;
+    P:809-811).  int32 in Z/2^32; float32 input (or the fp64
+    output of a previous stage) evaluated in fp64 with fp32-rounded
+    coefficients."""
+    lib = _load()
+    if dtype == "int32":
+        x = np.ascontiguousarray(x, dtype=np.int32)
+        y = np.empty_like(x)
+        ai, bi = _int_coeffs(a), _int_coeffs(b)
+        lib.oracle_rev_i32(_ptr(x), _ptr(y), x.shape[0], _ptr(ai), len(a) - 1, _ptr(bi) if len(bi) else None, len(bi))
+        return y
+    if dtype == "float32":
+        xd = np.ascontiguousarray(x, dtype=np.float64)
+        y = np.empty_like(xd)
+        af, bf = f32c(a), f32c(b)
+        lib.oracle_rev_f64(_ptr(xd), _ptr(y), xd.shape[0], _ptr(af), len(a) - 1, _ptr(bf) if len(bf) else None, len(bf))
+        return y
+    raise ValueError(dtype)
+
+
+def bidirectional(x, a, b, dtype: str) -> np.ndarray:
+    """Forward-backward (zero-phase) filtering: the anticausal recurrence of
+    the causal one's output (intermediate unrounded for float32)."""
+    return anticausal(recurrence(x, a, b, dtype), a, b, dtype)
 
 
 def factor_lists(b, m: int, dtype: str) -> np.ndarray:

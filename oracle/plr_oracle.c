@@ -138,6 +138,35 @@ void oracle_eq1_f64_dd(const double* x, double* y, int64_t n,
     }
 }
 
+/* The anticausal recurrence: Eq. (1) with the time direction reversed,
+ *   y_i = sum_{j=0..p} a_{-j} x_{i+j} + sum_{j=1..k} b_{-j} y_{i+j},
+ * x_j = y_j = 0 for j >= n, evaluated from i = n-1 down to 0 -- the backward
+ * filter of the causal/anticausal pairs of P:809-811 and P:866-868.  Same
+ * arithmetic as oracle_eq1_i32 (Z/2^32) and oracle_eq1_f64_dd (fp64). */
+void oracle_rev_i32(const int32_t* x, int32_t* y, int64_t n, const int64_t* a, int p, const int64_t* b, int k)
+{
+    for (int64_t i = n - 1; i >= 0; i--) {
+        uint64_t acc = 0;
+        for (int j = 0; j <= p; j++)
+            if (i + j < n) acc += (uint64_t)a[j] * (uint64_t)(uint32_t)x[i + j];
+        for (int j = 1; j <= k; j++)
+            if (i + j < n) acc += (uint64_t)b[j - 1] * (uint64_t)(uint32_t)y[i + j];
+        y[i] = (int32_t)(uint32_t)(acc & 0xffffffffu);
+    }
+}
+
+void oracle_rev_f64(const double* x, double* y, int64_t n, const double* a, int p, const double* b, int k)
+{
+    for (int64_t i = n - 1; i >= 0; i--) {
+        double acc = 0.0;
+        for (int j = 0; j <= p; j++)
+            if (i + j < n) acc += a[j] * x[i + j];
+        for (int j = 1; j <= k; j++)
+            if (i + j < n) acc += b[j - 1] * y[i + j];
+        y[i] = acc;
+    }
+}
+
 /* ---------------------------------------------------------------------- */
 /* Correction-factor lists (Sec. 2.1)                            */
 /* ---------------------------------------------------------------------- */

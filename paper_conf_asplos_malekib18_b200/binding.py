@@ -30,6 +30,8 @@ _SIGS = {
     "plr_plan_debug_stats": ([_P, _P, _I], _st),
     "plr_execute": ([_P, _P, _P, _S, _P], _st),
     "plr_execute_continue": ([_P, _P, _P, _S, _P, _P, _P], _st),
+    "plr_execute_reverse": ([_P, _P, _P, _S, _P], _st),
+    "plr_execute_bidirectional": ([_P, _P, _P, _S, _P, _P], _st),
     "plr_reduce": ([_P, _P, _S, _P, _P], _st),
     "plr_payload_from_output": ([_P, _P, _P, _S, _P, _P], _st),
     "plr_combine": ([_P, _P, _I, _I, _P, _P], _st),
@@ -247,6 +249,27 @@ class Plan:
         n = x.numel()
         _check(lib.plr_execute(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), n, _stream_ptr(stream)),
                "plr_execute")
+        return out
+
+    def reverse(self, x, out=None, stream=None):
+        """The anticausal recurrence (Eq. (1) from the end, zero beyond it)."""
+        out = self._out(x, out)
+        _check(lib.plr_execute_reverse(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), x.numel(),
+                                       _stream_ptr(stream)), "plr_execute_reverse")
+        return out
+
+    def bidirectional(self, x, out=None, tmp=None, stream=None):
+        """Forward then backward (zero-phase) filtering; tmp holds the forward
+        result (allocated when p > 0 and not given)."""
+        out = self._out(x, out)
+        if tmp is None and self.p > 0:
+            tmp = _torch().empty_like(x)
+        if tmp is not None and tmp.numel() != x.numel():
+            raise ValueError("tmp must have x.numel() elements")
+        self._on_plan_device(tmp)
+        _check(lib.plr_execute_bidirectional(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), x.numel(),
+                                             _dev_ptr(tmp, self.dtype) if tmp is not None else None,
+                                             _stream_ptr(stream)), "plr_execute_bidirectional")
         return out
 
     def continue_(self, x, out=None, x_hist=None, y_hist=None, stream=None):

@@ -234,7 +234,7 @@ AugMat<R> aug_matrix(const PlanTables& pt) {
 
 // ============================================================ launches ====
 static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const void* x_hist,
-                         const void* y_hist, void* y_tail, bool store, cudaStream_t stream) {
+                         const void* y_hist, void* y_tail, bool store, cudaStream_t stream, bool reverse = false) {
     if (n == 0) return PLR_OK;
     if (n > plan->n_max) return fail(PLR_ERR_SIZE, "n exceeds the plan's n_max");
     if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
@@ -243,7 +243,9 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         plan->epoch = 0;
         plan->dirty = false;
     }
-    if (n <= plan->small_max) {                 // small n: one CTA per tile, no pipeline
+    // small n: one CTA per tile, no pipeline; the anticausal pass of a
+    // non-DECAY plan runs the small-n kernel at every size
+    if (n <= plan->small_max || (reverse && !plan->pt.decay_flag)) {
         const uint64_t ms = (uint64_t)plan->pt.geo_s.tile();
         plan->epoch++;
         LaunchArgs la;
@@ -258,6 +260,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         la.stats = plan->d_stats;
         la.grid = (int)la.ntiles;
         la.store = store;
+        la.reverse = reverse;
         la.stream = stream;
         cudaError_t e = launch_small(plan->pt, la);
         if (e != cudaSuccess) {
@@ -291,6 +294,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.sig = plan->sig_kernel ? plan->pt.sig_id : 0;
     la.store = store;
     la.unit1 = unit1;
+    la.reverse = reverse;
     la.stream = stream;
     cudaError_t e = launch_scan(plan->pt, la);
     if (e != cudaSuccess) {
@@ -429,7 +433,9 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default()) : 0;
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
-    plan->max_tiles = std::max<uint64_t>(plan->max_tiles, (plan->small_max + ms - 1) / ms);   // status slots cover both
+    // status slots cover the small-n tiles up to n_max: the anticausal pass of
+    // a non-DECAY plan runs the small-n kernel at every size
+    plan->max_tiles = std::max<uint64_t>(plan->max_tiles, (n_max + ms - 1) / ms);
     if (plan->max_tiles > (1ull << 31)) { plr_plan_destroy(plan); return fail(PLR_ERR_SIZE, "n_max too large"); }
     plan->status_slots = 1;
     while (plan->status_slots < plan->max_tiles) plan->status_slots <<= 1;
@@ -573,6 +579,28 @@ plr_status plr_execute(plr_plan* plan, const void* x, void* y, size_t n, void* s
     plr_status st = check_xy(plan, x, y, n, true);
     if (st != PLR_OK || n == 0) return st;
     return launch(plan, x, y, n, nullptr, nullptr, nullptr, true, (cudaStream_t)stream);
+}
+
+plr_status plr_execute_reverse(plr_plan* plan, const void* x, void* y, size_t n, void* stream) {
+    plr_status st = check_xy(plan, x, y, n, true);
+    if (st != PLR_OK || n == 0) return st;
+    return launch(plan, x, y, n, nullptr, nullptr, nullptr, true, (cudaStream_t)stream, true);
+}
+
+plr_status plr_execute_bidirectional(plr_plan* plan, const void* x, void* y, size_t n, void* tmp, void* stream) {
+    plr_status st = check_xy(plan, x, y, n, true);
+    if (st != PLR_OK || n == 0) return st;
+    if (tmp == nullptr && plan->pt.p > 0)
+        return fail(PLR_ERR_INVALID_ARG, "p > 0: the forward pass needs a tmp buffer (the reverse pass cannot run in place)");
+    void* mid = tmp != nullptr ? tmp : y;
+    if (tmp != nullptr) {
+        if ((st = check_xy(plan, x, tmp, n, true)) != PLR_OK) return st;
+        if ((st = check_xy(plan, tmp, y, n, true)) != PLR_OK) return st;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    st = launch(plan, x, mid, n, nullptr, nullptr, nullptr, true, s, false);        // causal pass
+    if (st != PLR_OK) return st;
+    return launch(plan, mid, y, n, nullptr, nullptr, nullptr, true, s, true);        // anticausal pass
 }
 
 plr_status plr_execute_continue(plr_plan* plan, const void* x, void* y, size_t n, const void* x_hist,

@@ -574,8 +574,12 @@ struct Layout {
 // of SURVEY §8(a) a6) instead of correcting parked chunk values with the
 // factors h^(r)_u; the stage then holds the map outputs t (Eq. 2) between
 // the phases, or x itself when p = 0 (t = a0 x is recomputed).
+// REV: the anticausal recurrence (the causal one over the reversed
+// sequence; see plr_kernels_small.cuh): ticket j is original tile
+// ntiles-1-j read back to front, the ragged tile first (a virtual full tile,
+// zero beyond n), the map's halo after the tile; stage layout [tile][halo].
 template <typename T, typename A, int K, int P, int X, int W, int S, int D, int NL, bool DEC, bool STORE,
-          int MINB, bool SEED = false>
+          int MINB, bool SEED = false, bool REV = false>
 __global__ void __launch_bounds__((W + 1 + NL) * 32, MINB)
 plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = Layout<T, A, K, X, W, S, D>;
@@ -612,6 +616,13 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
     const Tables<T, A>& tb = prm.tab;
+    static_assert(!REV || STORE, "the anticausal pass always stores");
+    // the tile the compute warps load element by element (REV: the first)
+    auto is_ragged = [&](long long j) -> bool { return last_ragged && j == (REV ? 0 : ntiles - 1); };
+    // first element of tile j in the arrays (REV: original tile ntiles-1-j)
+    auto tile_start = [&](long long j) -> long long { return (REV ? ntiles - 1 - j : j) * (long long)M; };
+    // the tile's M words inside a stage ([halo][tile], REV: [tile][halo])
+    auto tile_words = [&](T* st) -> T* { return REV ? st : st + kHalo; };
 
     // launch state from device memory (tickets, epoch); the barrier consumes
     // the loads, so they complete before this CTA's first ticket grab
@@ -646,9 +657,18 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 launch_state_advance(prm.ticket, j, (unsigned long long)ntiles + gridDim.x, tbase, epoch);
                 stop_at = idx; mbar_arrive(&full_bar[s]); return;
             }
-            if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_bar[s]); return; }   // compute loads it
+            if (is_ragged(j)) { mbar_arrive(&full_bar[s]); return; }   // compute loads it
             T* st = stages + (size_t)s * SW;
-            if (j == 0) {
+            if (REV) {                                  // the tile, its halo after it (zero beyond n)
+                const long long o = tile_start(j);
+#pragma unroll
+                for (int q = 0; q < kHalo; q++) {
+                    const unsigned long long i = (unsigned long long)(o + M + q);
+                    st[M + q] = (q < P && i < n) ? prm.x[i] : T(0);
+                }
+                mbar_arrive_tx(&full_bar[s], M * sizeof(T));
+                bulk_load(st, prm.x + (size_t)o, M * sizeof(T), &full_bar[s], pol);
+            } else if (j == 0) {
 #pragma unroll
                 for (int q = 0; q < kHalo; q++)
                     st[q] = (q >= kHalo - P && prm.x_hist != nullptr) ? prm.x_hist[q - (kHalo - P)] : T(0);
@@ -668,8 +688,8 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (j >= ntiles) break;
             mbar_wait(&done_bar[s], (uint32_t)((it / S) & 1));
             bool stored = false;
-            if (STORE && !(j == ntiles - 1 && last_ragged)) {
-                bulk_store(prm.y + (size_t)j * M, stages + (size_t)s * SW + kHalo, M * sizeof(T), pol);
+            if (STORE && !is_ragged(j)) {
+                bulk_store(prm.y + (size_t)tile_start(j), tile_words(stages + (size_t)s * SW), M * sizeof(T), pol);
                 bulk_commit();
                 stored = true;
             }
@@ -780,13 +800,26 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (tid == 0) { agg_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
             return j;
         }
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         T* st = stages + (size_t)s * SW;
         const long long g0 = j * (long long)M + (long long)tid * X;
 
         // a1: my X elements (+ P halo), FIR map in the data type
         T xv[X + P];
-        if (!ragged) {
+        if (REV) {                                              // positions v: element o + M-1-v
+            const int v0 = tid * X - P;
+            if (!ragged) {
+#pragma unroll
+                for (int q = 0; q < X + P; q++) xv[q] = st[M - 1 - (v0 + q)];
+            } else {
+                const long long o = tile_start(j);
+#pragma unroll
+                for (int q = 0; q < X + P; q++) {
+                    const unsigned long long i = (unsigned long long)(o + M - 1 - (v0 + q));
+                    xv[q] = i < n ? prm.x[i] : T(0);
+                }
+            }
+        } else if (!ragged) {
             const T* base = st + kHalo + tid * X;
 #pragma unroll
             for (int q = 0; q < P; q++) xv[q] = base[q - P];
@@ -856,7 +889,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         // recomputed), except for the ragged tile the compute warps loaded
         if (!SEED || P > 0 || ragged) {
 #pragma unroll
-            for (int u = 0; u < X; u++) st[kHalo + tid * X + u] = lf[u];
+            for (int u = 0; u < X; u++) st[REV ? M - 1 - (tid * X + u) : kHalo + tid * X + u] = lf[u];
         }
 
         // a4, DECAY with T(32X d) == 0 for d >= 1 (dec_mask bit 5 clear): the
@@ -920,8 +953,10 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         const int s = it % S;
         const int slot = it % NS;
         mbar_wait(&carry_bar[slot], (uint32_t)((it / NS) & 1));
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         T* st = stages + (size_t)s * SW;
+        // the stage word of the thread's element u (REV: mirrored, original order)
+        auto at = [&](int u) -> T& { return st[REV ? M - 1 - (tid * X + u) : kHalo + tid * X + u]; };
         const long long g0 = j * (long long)M + (long long)tid * X;
         A Gp[K], Win[K], Sst[K];
 #pragma unroll
@@ -947,14 +982,13 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         T Sd[K];
 #pragma unroll
         for (int q = 0; q < K; q++) Sd[q] = cvt<T, A>(Sst[q]);
-        T* base = st + kHalo + tid * X;
         T yv[X];
         if constexpr (SEED) {
             // a6: y_u = t_u + sum_r b-r y_{u-r}, seeded with Sd = (y_{-1}, ..., y_{-K})
             const bool has_t = P > 0 || ragged;
 #pragma unroll
             for (int u = 0; u < X; u++) {
-                T acc = has_t ? base[u] : tb.alpha[0] * base[u];
+                T acc = has_t ? at(u) : tb.alpha[0] * at(u);
 #pragma unroll
                 for (int r = K; r >= 1; r--) acc = mad(tb.cT[r - 1], Sd[r - 1], acc);
 #pragma unroll
@@ -965,7 +999,7 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         } else {
 #pragma unroll
             for (int u = 0; u < X; u++) {
-                T acc = base[u];
+                T acc = at(u);
 #pragma unroll
                 for (int r = 0; r < K; r++) acc = mad(tb.H[u][r], Sd[r], acc);
                 yv[u] = acc;
@@ -974,16 +1008,16 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         if (!ragged) {
             if (STORE) {
 #pragma unroll
-                for (int u = 0; u < X; u++) base[u] = yv[u];
+                for (int u = 0; u < X; u++) at(u) = yv[u];
             }
         } else if (STORE) {
 #pragma unroll
             for (int u = 0; u < X; u++) {
-                const long long i = g0 + u;
+                const long long i = REV ? tile_start(j) + M - 1 - (tid * X + u) : g0 + u;
                 if ((unsigned long long)i < n) prm.y[i] = yv[u];
             }
         }
-        if (prm.y_tail != nullptr) {
+        if (!REV && prm.y_tail != nullptr) {
             const long long lo = (long long)n - K;
             if (g0 + X > lo && g0 < (long long)n) {
 #pragma unroll

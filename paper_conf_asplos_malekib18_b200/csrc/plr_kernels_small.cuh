@@ -20,6 +20,15 @@
 //   scan (one warp), a5 decoupled look-back of the k carries by warp 0 (the
 //   single hop of DECAY plans, T(m) = 0), a6 seeded serial recurrence from
 //   the true incoming state, a7 store.
+//
+// REV: the anticausal recurrence y_i = sum_j a_j x_{i+j} + sum_j b_j y_{i+j}
+// (zero beyond the end): the causal one over the reversed sequence, the
+// other half of a forward-backward (zero-phase) filter pair (P:809-811,
+// P:866-868).  Ticket j processes ORIGINAL tile o = ntiles-1-j, read back to
+// front, so tiles stay 16-byte aligned; the ragged last tile comes first,
+// as a full virtual tile whose positions beyond n are zero (zero inputs
+// before the start leave the zero state unchanged), and the map's halo
+// lies after the tile instead of before it.
 #pragma once
 #include "plr_kernels.cuh"
 
@@ -38,7 +47,7 @@ struct LayoutS {
     static constexpr size_t bytes = off_tile + 8;
 };
 
-template <typename T, typename A, int K, int P, int X, int W>
+template <typename T, typename A, int K, int P, int X, int W, bool REV = false>
 __global__ void __launch_bounds__(W * 32, 2)
 plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = LayoutS<T, A, K, X, W>;
@@ -77,10 +86,19 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         s_epoch = epoch;
         mbar_init(bar, 1);
         fence_mbar_init();
-        const bool ragged_ = (unsigned long long)(j + 1) * M > n;
+        const bool ragged_ = REV ? (j == 0 && n % (unsigned long long)M != 0) : (unsigned long long)(j + 1) * M > n;
         if (!ragged_) {                              // one TMA bulk load of the tile (+ halo)
             const uint64_t pol = policy_evict_first();
-            if (j == 0) {
+            if (REV) {                               // original tile o, halo after it (zero beyond n)
+                const long long o = ntiles - 1 - j;
+#pragma unroll
+                for (int q = 0; q < kHalo; q++) {
+                    const unsigned long long i = (unsigned long long)(o + 1) * M + q;
+                    stage[M + q] = (q < P && i < n) ? prm.x[i] : T(0);
+                }
+                mbar_arrive_tx(bar, M * sizeof(T));
+                bulk_load(stage, prm.x + (size_t)o * M, M * sizeof(T), bar, pol);
+            } else if (j == 0) {
 #pragma unroll
                 for (int q = 0; q < kHalo; q++)
                     stage[q] = (q >= kHalo - P && prm.x_hist != nullptr) ? prm.x_hist[q - (kHalo - P)] : T(0);
@@ -96,12 +114,27 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const long long j = *s_tile;
     const uint32_t epoch = s_epoch;
     const uint32_t tagA = 2u * epoch, tagI = 2u * epoch + 1u;
-    const bool ragged = (unsigned long long)(j + 1) * M > n;
+    const bool ragged = REV ? (j == 0 && n % (unsigned long long)M != 0) : (unsigned long long)(j + 1) * M > n;
     const long long g0 = j * (long long)M + (long long)tid * X;
+    // REV: tile position v (processing order) is original element oM + M-1-v
+    const long long oM = REV ? (ntiles - 1 - j) * (long long)M : 0;
+    const int v0 = tid * X;
 
     // a1: my X inputs (+ P halo) and the map t (Eq. 2)
     T xv[X + P];
-    if (!ragged) {
+    if (REV) {
+        if (!ragged) {
+            mbar_wait(bar, 0);
+#pragma unroll
+            for (int q = 0; q < X + P; q++) xv[q] = stage[M - 1 - (v0 - P + q)];
+        } else {
+#pragma unroll
+            for (int q = 0; q < X + P; q++) {
+                const unsigned long long i = (unsigned long long)(oM + M - 1 - (v0 - P + q));
+                xv[q] = i < n ? prm.x[i] : T(0);
+            }
+        }
+    } else if (!ragged) {
         mbar_wait(bar, 0);
         const T* base = stage + kHalo + tid * X;
 #pragma unroll
@@ -261,7 +294,18 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     }
     // a7: y into the stage and one TMA bulk store (ragged tile: direct stores)
     const bool store = prm.y != nullptr;
-    if (!ragged) {
+    if (REV) {
+        if (!ragged) {
+#pragma unroll
+            for (int u = 0; u < X; u++) stage[M - 1 - (v0 + u)] = yv[u];
+        } else {
+#pragma unroll
+            for (int u = 0; u < X; u++) {
+                const unsigned long long i = (unsigned long long)(oM + M - 1 - (v0 + u));
+                if (i < n) prm.y[i] = yv[u];
+            }
+        }
+    } else if (!ragged) {
         if (store) {
             T* base = stage + kHalo + tid * X;
 #pragma unroll
@@ -274,7 +318,7 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if ((unsigned long long)i < n) prm.y[i] = yv[u];
         }
     }
-    if (prm.y_tail != nullptr) {
+    if (!REV && prm.y_tail != nullptr) {
         const long long lo = (long long)n - K;
         if (g0 + X > lo && g0 < (long long)n) {
 #pragma unroll
@@ -288,7 +332,8 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         fence_proxy_async();
         __syncthreads();
         if (tid == 0) {
-            bulk_store(prm.y + (size_t)j * M, stage + kHalo, M * sizeof(T), policy_evict_first());
+            if (REV) bulk_store(prm.y + (size_t)oM, stage, M * sizeof(T), policy_evict_first());
+            else bulk_store(prm.y + (size_t)j * M, stage + kHalo, M * sizeof(T), policy_evict_first());
             bulk_commit();
             bulk_wait_read<0>();                     // smem stays valid until the store has read it
         }

@@ -26,6 +26,7 @@ struct LaunchArgs {
     int sig = 0;                        // compile-time signature id (plr_constsig.cuh), 0 = runtime tables
     bool store;
     bool unit1 = false;                 // look-back units of one tile (small n): the *_u1 kernels
+    bool reverse = false;               // the anticausal recurrence (REV kernels: small-n, DECAY)
     cudaStream_t stream;
     int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel
 };

@@ -159,15 +159,21 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
         threads = (TC::W + 1 + TC::NL) * 32;
     } else {
         kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB, C::SEED>;
+        if constexpr (C::DEC && STORE) {                 // the anticausal pass (DECAY plans)
+            if (la.reverse)
+                kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB, C::SEED,
+                                             true>;
+        }
         smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
         threads = (C::W + 1 + C::NL) * 32;
     }
     // the > 48 KB dynamic shared memory opt-in is a per-device (context)
-    // attribute: one bit per device, set once (racing sets are idempotent)
+    // attribute: one bit per device and kernel, set once (racing sets are
+    // idempotent); bit 63 - dev: the reverse kernel
     static std::atomic<unsigned long long> configured{0};
     int dev = 0;
     if (cudaError_t e = cudaGetDevice(&dev); e != cudaSuccess) return e;
-    const unsigned long long bit = 1ull << (dev & 63);
+    const unsigned long long bit = 1ull << (la.reverse ? 63 - (dev & 31) : (dev & 31));
     if (!(configured.load(std::memory_order_acquire) & bit)) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;

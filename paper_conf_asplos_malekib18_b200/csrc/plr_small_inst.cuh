@@ -10,7 +10,8 @@ namespace small_inst {
 template <typename T, typename A, int K, int P>
 cudaError_t launch_kp(const Tables<T, A>& tab, const LaunchArgs& la) {
     using L = dev::LayoutS<T, A, K, kSmallX, kSmallW>;
-    void (*kern)(const ScanParams<T, A>) = &dev::plr_small_kernel<T, A, K, P, kSmallX, kSmallW>;
+    void (*kern)(const ScanParams<T, A>) = la.reverse ? &dev::plr_small_kernel<T, A, K, P, kSmallX, kSmallW, true>
+                                                      : &dev::plr_small_kernel<T, A, K, P, kSmallX, kSmallW, false>;
     static_assert(L::bytes <= 48 * 1024, "small-n kernel needs no dynamic shared memory opt-in");
     if (la.occupancy_out != nullptr)
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, kSmallW * 32, L::bytes);

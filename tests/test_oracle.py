@@ -337,3 +337,50 @@ def test_cascade_float_matches_scipy_composed():
     ref = signal.lfilter(num, den, x.astype(np.float64))
     y = oracle.cascade(x, stages, "float32")
     np.testing.assert_allclose(y, ref, rtol=1e-9, atol=1e-12)
+
+
+# ------------------------------------------------------------ anticausal ---
+def test_anticausal_closed_forms_on_ones():
+    """Backward prefix sums of ones: (1: 1) -> n - i, (1: 2, -1) -> C(n-i+1, 2)
+    (the binomial signatures of P:140-143, run from the end)."""
+    n = 5000
+    i = np.arange(n, dtype=np.int64)
+    x = np.ones(n, np.int32)
+    assert oracle.anticausal(x, (1,), (1,), "int32").tolist() == (n - i).tolist()
+    assert oracle.anticausal(x, (1,), (2, -1), "int32").tolist() == ((n - i + 1) * (n - i) // 2).tolist()
+
+
+def test_anticausal_is_time_reversal_of_causal():
+    """Reversing time maps the anticausal recurrence onto Eq. (1): checked
+    against the causal oracle on reversed full-range / float inputs."""
+    for dtype, a, b in (("int32", (3, -1, 2), (2, -1)), ("float32", (0.729, -2.187, 2.187, -0.729), (2.4, -1.92, 0.512))):
+        x = workloads.host_input(3000, dtype, 8)
+        y = oracle.anticausal(x, a, b, dtype)
+        r = oracle.recurrence(x[::-1].copy(), a, b, dtype)[::-1]
+        if dtype == "int32":
+            assert np.array_equal(y, r)
+        else:
+            np.testing.assert_allclose(y, r, rtol=1e-12, atol=1e-12)
+
+
+def test_bidirectional_lp1_impulse_is_symmetric_closed_form():
+    """Zero-phase LP1: an impulse far from both ends gives
+    z_i = a^2 r^|i-c| / (1 - r^2) (the autocorrelation of a r^i), symmetric
+    about the impulse; a, r the fp32-rounded 0.2 and 0.8."""
+    n, c = 2000, 1000
+    x = np.zeros(n, np.float32)
+    x[c] = 1
+    z = oracle.bidirectional(x, (0.2,), (0.8,), "float32")
+    a, r = float(np.float32(0.2)), float(np.float32(0.8))
+    i = np.arange(n)
+    sel = np.abs(i - c) < 300
+    np.testing.assert_allclose(z[sel], (a * a * r ** np.abs(i - c) / (1 - r * r))[sel], rtol=1e-9, atol=1e-15)
+
+
+def test_bidirectional_prefix_closed_form():
+    """Forward then backward prefix sum of ones: sum_{j>=i} (j+1) =
+    (n(n+1) - i(i+1)) / 2, mod 2^32."""
+    n = 100000
+    i = np.arange(n, dtype=object)
+    z = oracle.bidirectional(np.ones(n, np.int32), (1,), (1,), "int32")
+    assert z.tolist() == [wrap32(int(v)) for v in (n * (n + 1) - i * (i + 1)) // 2]
