@@ -119,6 +119,44 @@ class ClockSampler:
                 "sm_max_mhz": self.max_mhz, "reasons": rs, "samples": len(self.samples)}
 
 
+# ----------------------------------------------------------- host CPU info --
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
+class PinnedCore:
+    """Pin this process to one host core while the single-threaded oracle is
+    timed (`taskset -c 0`; Eq. (1) is a loop-carried
+    dependence), then restore the affinity."""
+
+    def __init__(self, core=0):
+        self.core = core
+        self.old = None
+
+    def __enter__(self):
+        try:
+            self.old = os.sched_getaffinity(0)
+            os.sched_setaffinity(0, {self.core})
+        except Exception:
+            self.old = None
+        return self
+
+    def __exit__(self, *a):
+        if self.old is not None:
+            os.sched_setaffinity(0, self.old)
+
+    def desc(self):
+        return "pinned to host core %d (sched_setaffinity, as taskset -c %d)" % (self.core, self.core) \
+            if self.old is not None else "not pinned (sched_setaffinity unavailable)"
+
+
 # --------------------------------------------------------------- reference --
 def run_reference(args, rank, world):
     import numpy as np
@@ -130,19 +168,22 @@ def run_reference(args, rank, world):
     for name in WORKLOAD_SIGS:
         sig = workloads.BY_NAME[name]
         xs[name] = workloads.host_input(sample, sig.dtype, workloads.seed_for(1))
-    for _ in range(args.warmup):
-        for name in WORKLOAD_SIGS:
-            sig = workloads.BY_NAME[name]
-            oracle.recurrence(xs[name], sig.a, sig.b, sig.dtype)
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        for name in WORKLOAD_SIGS:
-            sig = workloads.BY_NAME[name]
-            oracle.recurrence(xs[name], sig.a, sig.b, sig.dtype)
-    dt = time.perf_counter() - t0
+    pin = PinnedCore(0)
+    with pin:
+        for _ in range(args.warmup):
+            for name in WORKLOAD_SIGS:
+                sig = workloads.BY_NAME[name]
+                oracle.recurrence(xs[name], sig.a, sig.b, sig.dtype)
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            for name in WORKLOAD_SIGS:
+                sig = workloads.BY_NAME[name]
+                oracle.recurrence(xs[name], sig.a, sig.b, sig.dtype)
+        dt = time.perf_counter() - t0
     elems = args.steps * sample * len(WORKLOAD_SIGS)
     gbs = elems * BYTES_PER_ELT / dt / 1e9
-    desc = "first 2^24 elements of the workload input per signature per step, sequential C oracle (gcc -O2), 1 thread"
+    desc = ("first 2^24 elements of the workload input per signature per step, sequential C oracle (gcc -O2), "
+            "1 thread, %s" % pin.desc())
     line = {
         "impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 3),
@@ -150,7 +191,8 @@ def run_reference(args, rank, world):
         "data": "synthetic (seeded uniform int32)",
         "config": {"workload": "configs[1] tuple prefix sums (1:0,1)+(1:0,0,1), bounded sample", "n_per_sig": sample},
         "elements_per_s": elems / dt,
-        "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc},
+        "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc,
+                         "cpu_model": cpu_model(), "host_cores_available": os.cpu_count()},
         "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -246,6 +288,9 @@ def main():
                        "n_per_gpu": n, "signatures": [workloads.BY_NAME[s].text() for s in WORKLOAD_SIGS],
                        "l2": "inputs 4 GiB per tensor >> 126 MB L2 (no flush needed)",
                        "tile_elems": plans[WORKLOAD_SIGS[0]].info["tile_elems"],
+                       "kernel_specialisation": "compile-time signature tables (plr_constsig.cuh: the paper's "
+                                                "per-signature code generation, P:640-649, P:721-729); const_sig=%d"
+                                                % plans[WORKLOAD_SIGS[0]].info["const_sig"],
                        "ctas_per_sm": plans[WORKLOAD_SIGS[0]].info["ctas_per_sm"]},
             "elements_per_s": elems_step / (ms_step * 1e-3),
             "frac_of_hbm_peak": round(gbs / world / hbm, 4),
@@ -377,16 +422,18 @@ def run_extras(args, plr, torch, np, n, x, y, plans, hbm):
     import oracle
     sample = min(n, 1 << 30)             # ~10 s of single-core work for both signatures
     xs = x[:sample].cpu().numpy()
-    t0 = time.perf_counter()
-    for name in WORKLOAD_SIGS:
-        sig = workloads.BY_NAME[name]
-        oracle.recurrence(xs, sig.a, sig.b, sig.dtype)
-    dt = time.perf_counter() - t0
+    pin = PinnedCore(0)
+    with pin:
+        t0 = time.perf_counter()
+        for name in WORKLOAD_SIGS:
+            sig = workloads.BY_NAME[name]
+            oracle.recurrence(xs, sig.a, sig.b, sig.dtype)
+        dt = time.perf_counter() - t0
     cg = sample * len(WORKLOAD_SIGS) * BYTES_PER_ELT / dt / 1e9
     out["cpu_baseline"] = {"value": round(cg, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
                            "sample": "first %d elements of the workload input, each of the 2 signatures, "
-                                     "sequential C oracle (gcc -O2), 1 thread, %.1f s" % (sample, dt),
-                           "host_cores_available": os.cpu_count()}
+                                     "sequential C oracle (gcc -O2), 1 thread, %.1f s, %s" % (sample, dt, pin.desc()),
+                           "cpu_model": cpu_model(), "host_cores_available": os.cpu_count()}
     return out
 
 
