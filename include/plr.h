@@ -174,6 +174,14 @@ plr_status plr_execute(plr_plan* plan, const void* x, void* y, size_t n, void* s
  * with the same hierarchy and look-back. */
 plr_status plr_execute_reverse(plr_plan* plan, const void* x, void* y, size_t n, void* stream);
 
+/* The paper's "Scan" comparator: Blelloch's
+ * (k x k matrix, k-vector) prefix-scan formulation of the same recurrence,
+ * through CUB DeviceScan, fp32 / Z/2^32 arithmetic, zero initial state.  A
+ * comparison baseline for benchmarks, NOT the PLR
+ * path.  Same arguments and rules as plr_execute; the first call (and any
+ * larger n) allocates CUB's temporary storage in the plan (synchronously). */
+plr_status plr_scan_comparator(plr_plan* plan, const void* x, void* y, size_t n, void* stream);
+
 /* Forward-backward (zero-phase) filtering: y = reverse(forward(x)), i.e. the
  * causal recurrence then the anticausal one (plr_execute_reverse) on its
  * output, two passes.  tmp (device, n elements of the dtype) holds the

@@ -31,6 +31,7 @@ _SIGS = {
     "plr_execute": ([_P, _P, _P, _S, _P], _st),
     "plr_execute_continue": ([_P, _P, _P, _S, _P, _P, _P], _st),
     "plr_execute_reverse": ([_P, _P, _P, _S, _P], _st),
+    "plr_scan_comparator": ([_P, _P, _P, _S, _P], _st),
     "plr_execute_bidirectional": ([_P, _P, _P, _S, _P, _P], _st),
     "plr_reduce": ([_P, _P, _S, _P, _P], _st),
     "plr_payload_from_output": ([_P, _P, _P, _S, _P, _P], _st),
@@ -256,6 +257,14 @@ class Plan:
         out = self._out(x, out)
         _check(lib.plr_execute_reverse(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), x.numel(),
                                        _stream_ptr(stream)), "plr_execute_reverse")
+        return out
+
+    def scan_comparator(self, x, out=None, stream=None):
+        """The paper's Scan comparator (Blelloch matrix-vector scan via CUB;
+        a baseline, not the PLR path)."""
+        out = self._out(x, out)
+        _check(lib.plr_scan_comparator(self._h, _dev_ptr(x, self.dtype), _dev_ptr(out, self.dtype), x.numel(),
+                                       _stream_ptr(stream)), "plr_scan_comparator")
         return out
 
     def bidirectional(self, x, out=None, tmp=None, stream=None):

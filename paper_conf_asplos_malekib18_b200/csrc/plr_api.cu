@@ -50,6 +50,8 @@ struct plr_plan {
     size_t small_max = 0;               // n <= small_max: the small-n kernel (plr_kernels_small.cuh)
     int reduce_ctas = 0;                // CTAs per SM of the reduce-only kernel (0: not available)
     unsigned long long* d_rd = nullptr; // its per-CTA records (kStatusMaxBytes each)
+    void* d_scan_tmp = nullptr;         // CUB temp storage of the Scan comparator
+    size_t scan_tmp_bytes = 0;
     float* d_fix = nullptr;
     bool dirty = false;
     bool sig_kernel = false;            // launch the compile-time signature kernel (pt.sig_id)
@@ -348,6 +350,7 @@ plr_status plr_plan_destroy(plr_plan* plan) {
     cudaFree(plan->d_lane);
     cudaFree(plan->d_lane_s);
     cudaFree(plan->d_rd);
+    cudaFree(plan->d_scan_tmp);
     cudaFree(plan->d_fix);
     cudaFree(plan->d_send);
     cudaFree(plan->d_recv);
@@ -601,6 +604,34 @@ plr_status plr_execute_bidirectional(plr_plan* plan, const void* x, void* y, siz
     st = launch(plan, x, mid, n, nullptr, nullptr, nullptr, true, s, false);        // causal pass
     if (st != PLR_OK) return st;
     return launch(plan, mid, y, n, nullptr, nullptr, nullptr, true, s, true);        // anticausal pass
+}
+
+plr_status plr_scan_comparator(plr_plan* plan, const void* x, void* y, size_t n, void* stream) {
+    plr_status st = check_xy(plan, x, y, n, true);
+    if (st != PLR_OK || n == 0) return st;
+    if (n > plan->n_max) return fail(PLR_ERR_SIZE, "n exceeds the plan's n_max");
+    cudaStream_t s = (cudaStream_t)stream;
+    const PlanTables& pt = plan->pt;
+    float cf[kMaxK], af[kMaxP + 1];
+    for (int r = 0; r < pt.k; r++) cf[r] = (float)pt.b_d[r];
+    for (int j = 0; j <= pt.p; j++) af[j] = (float)pt.a_d[j];
+    auto run = [&](void* tmp, size_t& bytes) -> cudaError_t {
+        if (pt.dtype == PLR_INT32)
+            return blelloch_i32((const uint32_t*)x, (uint32_t*)y, (long long)n, pt.b_u, pt.k, pt.a_u, pt.p, tmp, bytes, s);
+        return blelloch_f32((const float*)x, (float*)y, (long long)n, cf, pt.k, af, pt.p, tmp, bytes, s);
+    };
+    size_t need = 0;
+    CUDA_TRY(run(nullptr, need), "Scan comparator size query");
+    if (need > plan->scan_tmp_bytes) {
+        cudaFree(plan->d_scan_tmp);
+        plan->d_scan_tmp = nullptr;
+        plan->scan_tmp_bytes = 0;
+        CUDA_TRY(cudaMalloc(&plan->d_scan_tmp, need), "alloc Scan comparator storage");
+        plan->scan_tmp_bytes = need;
+    }
+    size_t have = plan->scan_tmp_bytes;
+    CUDA_TRY(run(plan->d_scan_tmp, have), "Scan comparator");
+    return PLR_OK;
 }
 
 plr_status plr_execute_continue(plr_plan* plan, const void* x, void* y, size_t n, const void* x_hist,

@@ -66,6 +66,11 @@ cudaError_t small_occupancy(const PlanTables& pt, int* ctas_per_sm);
 // scratch (kStatusMaxBytes each), la.grid CTAs over contiguous tile ranges of
 // kRedX * kRedW * 32 elements, la.y_tail = the K end-state outputs
 cudaError_t launch_reduce(const PlanTables& pt, const LaunchArgs& la);
+// the Scan comparator (plr_blelloch.cuh); tmp == nullptr: size query
+cudaError_t blelloch_i32(const uint32_t* x, uint32_t* y, long long n, const uint32_t* c, int k, const uint32_t* alpha,
+                         int p, void* tmp, size_t& tmp_bytes, cudaStream_t s);
+cudaError_t blelloch_f32(const float* x, float* y, long long n, const float* c, int k, const float* alpha, int p,
+                         void* tmp, size_t& tmp_bytes, cudaStream_t s);
 cudaError_t reduce_occupancy(const PlanTables& pt, int* ctas_per_sm);
 cudaError_t launch_reduce_i32(const Tables<uint32_t, uint32_t>& tab, const LaunchArgs& la, int k, int p);
 cudaError_t launch_reduce_f64acc(const Tables<float, double>& tab, const LaunchArgs& la, int k, int p);
