@@ -569,12 +569,16 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     for (; nb < na; nb++) phaseB(nb);                           // drain
     // stop markers: the storer, and look-back warps waiting beyond the stop
     {
-        // wait for the stage as phase B of position nb would: with STORE =
-        // false the storer releases stages at once, so it may not have
-        // consumed position nb - ST yet; arriving early would complete
-        // full_T[sT] a phase ahead of its parity wait (a hang)
+        // STORE = false: the storer releases every stage at once, so it may
+        // not have consumed position nb - ST yet; arriving early would
+        // complete full_T[sT] a phase ahead of its parity wait (a hang), so
+        // wait for the stage as phase B of position nb would.  STORE = true:
+        // phase B(nb-1)'s own wait implies the storer consumed position
+        // nb-2 >= nb-ST, and waiting here would deadlock: the storer keeps
+        // up to ST-1 stages until a further arrival (a ragged last tile is
+        // released out of that order), which is this marker's.
         const int sT = nb % ST;
-        mbar_wait(&empty_T[sT], (uint32_t)(((nb / ST) & 1) ^ 1));
+        if constexpr (!STORE) mbar_wait(&empty_T[sT], (uint32_t)(((nb / ST) & 1) ^ 1));
         if (tid == 0) store_tile[sT] = ntiles;
         mbar_arrive(&full_T[sT]);
     }
