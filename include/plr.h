@@ -106,6 +106,10 @@ typedef struct {
                                   data type) or 64 (fp64, reading R16)       */
     double cond_bound;         /* float: the planner's a-priori error bound of fp32
                                   accumulation relative to the output scale (R16); 0 int */
+    double map_floor;          /* float: the error floor of ANY fp32-data evaluation (the map
+                                  rounds the input) relative to a Nyquist-frequency output
+                                  (reading R20); 0 int                        */
+    double nyquist_gain;       /* float: |H(-1)|, the gain at the Nyquist frequency; 0 int */
 } plr_plan_info;
 
 /* Create a plan.  a[0..p] = (a0, a-1, ..., a-p) (p = feed-forward order, so

@@ -63,7 +63,8 @@ class PlanInfo(ctypes.Structure):
                 ("threads_per_cta", _I), ("tile_elems", _I), ("stages", _I), ("decay_len", ctypes.c_int64),
                 ("fixup_len", ctypes.c_int64), ("n_max", _S), ("scratch_bytes", _S), ("ctas_per_sm", _I),
                 ("num_sms", _I), ("const_sig", _I),
-                ("tiles_per_unit", _I), ("kernel_kind", _I), ("acc_bits", _I), ("cond_bound", ctypes.c_double)]
+                ("tiles_per_unit", _I), ("kernel_kind", _I), ("acc_bits", _I), ("cond_bound", ctypes.c_double),
+                ("map_floor", ctypes.c_double), ("nyquist_gain", ctypes.c_double)]
 
 
 class PLRError(RuntimeError):

@@ -558,6 +558,8 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->kernel_kind = kernel_kind(plan->pt);
     info->acc_bits = (plan->pt.dtype == PLR_FLOAT32 && plan->pt.acc64) ? 64 : 32;
     info->cond_bound = plan->pt.dtype == PLR_FLOAT32 ? plan->pt.cond_bound : 0.0;
+    info->map_floor = plan->pt.dtype == PLR_FLOAT32 ? plan->pt.map_floor : 0.0;
+    info->nyquist_gain = plan->pt.dtype == PLR_FLOAT32 ? plan->pt.nyquist_gain : 0.0;
     return PLR_OK;
 }
 

@@ -82,7 +82,9 @@ struct PlanTables {
     int decay_flag;
     int acc64;                           // float: accumulate recurrence + carries in fp64
     uint32_t dec_mask;                   // ScanParams::dec_mask of the tables the plan launches with
-    double cond_bound;                   // eps32 * sum|a| * (sum|g|)^2 (float)
+    double cond_bound;                   // eps32 * sum|a| * (sum|g|)^2 / min(1, |H(-1)|) (float, R16)
+    double map_floor;                    // eps32 * sum|a| * sum|g| / min(1, |H(-1)|) (float, R20)
+    double nyquist_gain;                 // |H(-1)| = |A(-1)| / |B(-1)| (float)
     int sig_id;                          // compile-time signature kernel (plr_constsig.cuh), 0 = none
     Tables<uint32_t, uint32_t> ti;       // int32 ring
     Tables<float, float> tf;             // fp32, fp32 accumulation

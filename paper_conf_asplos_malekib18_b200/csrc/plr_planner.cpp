@@ -297,6 +297,11 @@ plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype
         for (int j = 1; j <= k; j++) bn -= (j & 1) ? -c[j - 1] : c[j - 1];
         const double nyq = bn != 0.0 ? std::fabs(an / bn) : 1.0;
         pt.cond_bound = std::ldexp(1.0, -24) * sa * sg * sg / std::fmin(1.0, nyq);
+        // R20: the floor every fp32-data evaluation (the serial one too) has
+        // relative to the output: the map's fp32 rounding of the input scale,
+        // amplified once by the recurrence, over the Nyquist gain
+        pt.map_floor = std::ldexp(1.0, -24) * sa * sg / std::fmin(1.0, nyq);
+        pt.nyquist_gain = nyq;
         pt.acc64 = (!decays || !(pt.cond_bound <= 1e-3)) ? 1 : 0;
         if (!pt.decay_flag) pt.acc64 = 1;      // multi-tile look-back kernels exist in fp64 accumulation only
         pt.dec_mask = 0x3fu;

@@ -117,14 +117,21 @@ struct Cfg {
     static constexpr int S = S_, D = D_, NL = NL_, X = X_, W = W_, MINB = MINB_;
     static constexpr bool DEC = DEC_, U1 = U1_, SEED = SEED_;
 };
-// DECAY kernels: phase B seeded with the true carry (PLR_DEC_SEED=0: the
-// correction y = l + sum_r S_r h^(r)_u, kept for comparison builds)
+// DECAY phase B (measured r03b at 2^30, fraction of copy): fp32 plans keep
+// the correction y = l + sum_r S_r h^(r)_u (independent FMAs; seeded: LP1
+// 0.99 -> 0.95, HP2 0.98 -> 0.95, the serial chain is exposed); fp64-
+// accumulation plans run the fp32 recurrence seeded with the fp64 carry
+// (no per-element fp64 -> fp32 conversion of l, no factor table: HP3 0.79 ->
+// 0.81)
 #ifndef PLR_DEC_SEED
-#define PLR_DEC_SEED 1
+#define PLR_DEC_SEED 0
+#endif
+#ifndef PLR_DEC64_SEED
+#define PLR_DEC64_SEED 1
 #endif
 using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true, false, PLR_DEC_SEED>;
 using CfgDec64 = Cfg<PLR_DEC64_S, PLR_DEC64_D, PLR_DEC64_NL, PLR_DEC64_X, PLR_DEC64_W, PLR_DEC64_MINB, true, false,
-                     PLR_DEC_SEED>;
+                     PLR_DEC64_SEED>;
 using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false>;
 using CfgGen1 = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false, true>;
 

@@ -181,3 +181,17 @@ def test_cascade_validation(stages, code):
     with pytest.raises(plr.PLRError) as e:
         plr.Plan.cascade(stages, "int32", n_max=0)
     assert e.value.status == code
+
+
+def test_map_floor_reading_r20():
+    """Reading R20: every Table-1 float row has an fp32-data floor
+    eps32 sum|a| sum|g| / min(1, |H(-1)|) below the 1e-4 bar, so the
+    worked example's (-1)^i (i+3) input is a fair parity input for all of
+    them; a filter with a zero at the Nyquist frequency has no finite floor."""
+    for s in workloads.TABLE1:
+        if s.dtype == "float32":
+            info = plr.Plan(s.a, s.b, s.dtype, n_max=0).info
+            assert info["map_floor"] <= 1e-4, (s.name, info["map_floor"])
+    lp3 = plr.Plan((0.008,), (2.4, -1.92, 0.512), "float32", n_max=0).info
+    assert lp3["nyquist_gain"] == pytest.approx(0.008 / 5.832, rel=1e-5)
+    assert plr.Plan((0.25, 0.5, 0.25), (0.8,), "float32", n_max=0).info["map_floor"] == float("inf")

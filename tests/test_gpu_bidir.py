@@ -50,12 +50,16 @@ def test_bidirectional_parity(cuda_plr, sig):
         yd = torch.empty_like(xd)
         plan.bidirectional(xd, out=yd)
         check(yd.cpu().numpy(), ref, sig.dtype, "%s bidirectional in place" % sig.name)
-    xa = workloads.structured_input("alternating", 7 * 3840 + 123, sig.dtype)
-    pa = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=len(xa))
-    check(pa.bidirectional(torch.from_numpy(xa).cuda()).cpu().numpy(),
-          oracle.bidirectional(xa, sig.a, sig.b, sig.dtype), sig.dtype, "%s bidirectional alternating" % sig.name)
+    # (-1)^i (i+3) where fp32 data can meet the bar (reading R20): the pair
+    # attenuates a Nyquist input twice, so the floor is map_floor / |H(-1)|
+    info = plan.info
+    if sig.dtype == "int32" or info["map_floor"] / min(1.0, info["nyquist_gain"]) <= 1e-4:
+        xa = workloads.structured_input("alternating", 7 * 3840 + 123, sig.dtype)
+        pa = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=len(xa))
+        check(pa.bidirectional(torch.from_numpy(xa).cuda()).cpu().numpy(),
+              oracle.bidirectional(xa, sig.a, sig.b, sig.dtype), sig.dtype, "%s bidirectional alternating" % sig.name)
+        pa.close()
     plan.close()
-    pa.close()
 
 
 def test_reverse_full_size_decay(cuda_plr):
