@@ -27,7 +27,8 @@ struct LayoutRd {
     static constexpr int SW = M + kHalo;
     static constexpr size_t off_stage = 0;                                        // S x SW (T)
     static constexpr size_t off_wagg = ((size_t)S * SW * sizeof(T) + 15) & ~(size_t)15;   // [2][W][kMaxK] A
-    static constexpr size_t off_bar = off_wagg + 2 * (size_t)W * kMaxK * sizeof(A);
+    static constexpr size_t off_acc = off_wagg + 2 * (size_t)W * kMaxK * sizeof(A);  // [kMaxK] A: the CTA's fold
+    static constexpr size_t off_bar = (off_acc + kMaxK * sizeof(A) + 15) & ~(size_t)15;
     static constexpr size_t bytes = off_bar + 2 * S * 8 + 16;                     // full[S], empty[S], flag
 };
 
@@ -78,6 +79,7 @@ plr_reduce_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     extern __shared__ __align__(128) unsigned char smem[];
     T* stages = reinterpret_cast<T*>(smem + L::off_stage);
     A* wagg = reinterpret_cast<A*>(smem + L::off_wagg);
+    A* sacc = reinterpret_cast<A*>(smem + L::off_acc);
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + L::off_bar);
     uint64_t* empty = full + S;
     int* s_last = reinterpret_cast<int*>(empty + S);
@@ -125,9 +127,13 @@ plr_reduce_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             }
         }
     } else {
-        A acc[K];                                                // warp 0: fold of the CTA's tile aggregates
+        // the fold of the CTA's tile aggregates lives in sacc; tile f's warp-
+        // aggregate scan and fold run in warp f mod W (ordered after tile
+        // f-1's fold by tile f's named barrier), so no warp idles the others
+        if (tid == 0) {
 #pragma unroll
-        for (int e = 0; e < K; e++) acc[e] = A(0);
+            for (int e = 0; e < K; e++) sacc[e] = A(0);
+        }
         for (int f = 0; f < nt; f++) {
             const int s = f % S;
             const long long j = t0 + f;
@@ -187,8 +193,11 @@ plr_reduce_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 for (int e = 0; e < K; e++) wg[warp * kMaxK + e] = v[e];
             }
             named_sync(1, NC);
-            // a4 (warp 0): tile aggregate, folded in order: acc = T(L) acc + A_tile
-            if (warp == 0) {
+            // a4 (warp f mod W): tile aggregate, folded in order: acc = T(L) acc + A_tile
+            if (warp == f % W) {
+                A acc[K];
+#pragma unroll
+                for (int e = 0; e < K; e++) acc[e] = sacc[e];
                 A u_[K];
 #pragma unroll
                 for (int e = 0; e < K; e++) u_[e] = lane < W ? wg[lane * kMaxK + e] : A(0);
@@ -209,16 +218,20 @@ plr_reduce_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     companion_pow<A, K>(tb.c, n - (unsigned long long)j * M, Tr);
                     matvec_acc<A, K>(At, Tr, acc);
                 }
+                __syncwarp();
+                if (lane == 0) {
 #pragma unroll
-                for (int e = 0; e < K; e++) acc[e] = At[e];
+                    for (int e = 0; e < K; e++) sacc[e] = At[e];
+                }
             }
         }
+        named_sync(1, NC);                                       // the last fold is in sacc
         // the CTA's record: its fold and its length in elements
         if (warp == 0 && lane == 0) {
             unsigned long long* rec = rd_record<A>(prm.status, blockIdx.x);
             A* ra = reinterpret_cast<A*>(rec);
 #pragma unroll
-            for (int e = 0; e < K; e++) ra[e] = acc[e];
+            for (int e = 0; e < K; e++) ra[e] = sacc[e];
             const unsigned long long len = nt == 0 ? 0ull
                 : (t1 == ntiles ? n - (unsigned long long)t0 * M : (unsigned long long)nt * M);
             rec[(kStatusMaxBytes / 8) - 1] = len;
