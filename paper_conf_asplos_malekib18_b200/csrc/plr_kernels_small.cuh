@@ -35,6 +35,15 @@
 namespace plr {
 namespace dev {
 
+// PLR_TRACE builds: globaltimer stamps of the launch's LAST tile (the end of
+// its critical path) into stats words 9..15 (plan made with PLR_STATS=1)
+#ifdef PLR_TRACE
+#define PLR_STAMP_LAST(i) do { if (prm.stats != nullptr && j == ntiles - 1) { unsigned long long t_; \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_)); prm.stats[i] = t_; } } while (0)
+#else
+#define PLR_STAMP_LAST(i) do { } while (0)
+#endif
+
 template <typename T, typename A, int K, int X, int W>
 struct LayoutS {
     static constexpr int M = 32 * W * X;
@@ -77,11 +86,19 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // grab with relative index ntiles - 1 is this launch's last; every CTA
     // reads the base before its own grab
     __shared__ uint32_t s_epoch;
+#ifdef PLR_TRACE
+    unsigned long long t_entry;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_entry));
+#endif
     if (tid == 0) {
         const unsigned long long tbase = ld_volatile_u64(prm.ticket + 1);
         const uint32_t epoch = (uint32_t)ld_volatile_u64(prm.ticket + 2) + 1u;
         const long long j = (long long)(atomicAdd(prm.ticket, 1ull) - tbase);
         launch_state_advance(prm.ticket, j, (unsigned long long)ntiles, tbase, epoch);
+#ifdef PLR_TRACE
+        if (prm.stats != nullptr && j == ntiles - 1) prm.stats[9] = t_entry;
+#endif
+        PLR_STAMP_LAST(10);
         *s_tile = j;
         s_epoch = epoch;
         mbar_init(bar, 1);
@@ -125,6 +142,7 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     if (REV) {
         if (!ragged) {
             mbar_wait(bar, 0);
+            if (tid == 0) PLR_STAMP_LAST(11);
 #pragma unroll
             for (int q = 0; q < X + P; q++) xv[q] = stage[M - 1 - (v0 - P + q)];
         } else {
@@ -136,6 +154,7 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         }
     } else if (!ragged) {
         mbar_wait(bar, 0);
+        if (tid == 0) PLR_STAMP_LAST(11);
         const T* base = stage + kHalo + tid * X;
 #pragma unroll
         for (int q = 0; q < P; q++) xv[q] = base[q - P];
@@ -193,6 +212,7 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         for (int q = 0; q < K; q++) wagg[warp * kMaxK + q] = v[q];
     }
     __syncthreads();                                 // wagg complete; every stage read done
+    if (tid == 0) PLR_STAMP_LAST(12);
 
     // a4 + a5 (warp 0): warp-aggregate scan, publish, look back, publish
     if (warp == 0) {
@@ -244,6 +264,7 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             __syncwarp();
             lbs.flush(prm.stats, lane);
         }
+        if (lane == 0) PLR_STAMP_LAST(13);
         if (!decay || j == 0) {
             A G[K];
 #pragma unroll
@@ -331,11 +352,13 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     if (!ragged && store) {
         fence_proxy_async();
         __syncthreads();
+        if (tid == 0) PLR_STAMP_LAST(14);
         if (tid == 0) {
             if (REV) bulk_store(prm.y + (size_t)oM, stage, M * sizeof(T), policy_evict_first());
             else bulk_store(prm.y + (size_t)j * M, stage + kHalo, M * sizeof(T), policy_evict_first());
             bulk_commit();
             bulk_wait_read<0>();                     // smem stays valid until the store has read it
+            PLR_STAMP_LAST(15);
         }
     }
 }

@@ -1,5 +1,6 @@
-"""Critical path of CTA 0 in one small launch of the re-read kernel: globaltimer
-stamps (PLR_TRACE variant build, PLR_STATS=1), ns after the init barrier.
+"""Critical path of the LAST tile of one small-n launch (plr_kernels_small.cuh):
+globaltimer stamps (PLR_TRACE variant build, PLR_STATS=1), ns after that
+CTA's entry, median of 5 launches, L2 flushed before each.
 Usage: PLR_LIB=.../libplr_b200_trace.so python tools/trace_small.py"""
 import json
 import os
@@ -10,20 +11,24 @@ import torch  # noqa: E402
 import paper_conf_asplos_malekib18_b200 as plr  # noqa: E402
 import workloads  # noqa: E402
 
-NAMES = ["init", "entry", "lookback_unit0_done", "lookback_warp_exit", "storer_saw_stop", "storer_exit", "compute_end"]
-for name in ["tuple2", "order3"]:
-    for n in [1024, 7936 * 4, 1 << 20, 1 << 22]:
+NAMES = ["entry", "ticket", "loaded", "phaseA_sync", "lookback_done", "phaseB_done", "store_read"]
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+for name in ["prefix", "tuple2", "order3", "lp1", "hp3"]:
+    for n in [1 << 14, 1 << 18, 1 << 20, 1 << 22]:
         sig = workloads.BY_NAME[name]
         x = workloads.device_input(n, sig.dtype, 1)
         y = torch.empty_like(x)
         plan = plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
         rows = []
-        for r in range(6):
+        for r in range(7):
+            flush.fill_(r)
+            torch.cuda.synchronize()
             plan(x, y)
             torch.cuda.synchronize()
             t = plan.debug_stats(reset=True)["trace"]
             if r >= 2:
                 rows.append([(v - t[0]) if v else -1 for v in t])
         med = [sorted(c)[len(c) // 2] for c in zip(*rows)]
-        print(json.dumps({"sig": name, "n": n, "ns_after_init": dict(zip(NAMES, med))}), flush=True)
+        print(json.dumps({"sig": name, "n": n, "tiles": -(-n // plan.info["tile_elems"]) if False else None,
+                          "ns_after_entry": dict(zip(NAMES, med))}), flush=True)
         plan.close()
