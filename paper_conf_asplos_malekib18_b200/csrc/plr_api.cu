@@ -48,6 +48,7 @@ struct plr_plan {
     void* d_lane = nullptr;
     void* d_lane_s = nullptr;           // lane table T(X_s l) of the small-n kernel
     size_t small_max = 0;               // n <= small_max: the small-n kernel (plr_kernels_small.cuh)
+    int small_ctas = 0;                 // its CTAs per SM (all tiles resident: tile = blockIdx.x)
     int reduce_ctas = 0;                // CTAs per SM of the reduce-only kernel (0: not available)
     unsigned long long* d_rd = nullptr; // its per-CTA records (kStatusMaxBytes each)
     void* d_scan_tmp = nullptr;         // CUB temp storage of the Scan comparator
@@ -257,6 +258,13 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         la.status_mask = plan->status_slots - 1;
         la.decay = plan->pt.decay_s;
         la.dec_mask = plan->pt.dec_mask_s;
+        // every tile resident at once (one wave): tile index = blockIdx.x, no
+        // ticket before the load (PLR_SMALL_RESIDENT=0 turns it off)
+        static const bool resident_ok = [] {
+            const char* e = std::getenv("PLR_SMALL_RESIDENT");
+            return e == nullptr || e[0] != '0';
+        }();
+        if (resident_ok && la.ntiles <= (uint64_t)plan->num_sms * plan->small_ctas) la.dec_mask |= 0x100u;
         la.x_hist = x_hist; la.y_hist = y_hist; la.y_tail = y_tail;
         la.lane_T = plan->d_lane_s;
         la.stats = plan->d_stats;
@@ -434,6 +442,7 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
         }
     }
     plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default()) : 0;
+    plan->small_ctas = small_ctas;
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
     // status slots cover the small-n tiles up to n_max: the anticausal pass of

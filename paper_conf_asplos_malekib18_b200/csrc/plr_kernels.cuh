@@ -411,7 +411,8 @@ struct LbStats {
 template <typename T, typename A, int K, bool DEC>
 __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, const Tables<T, A>& tb, long long j,
                                                  int lane, uint32_t tagA, uint32_t tagI, A (&Gp)[K],
-                                                 const LbStats& lbs, long long c_start = 0, long long c_agg = 0) {
+                                                 const LbStats& lbs, long long c_start = 0, long long c_agg = 0,
+                                                 int ns_cap = 512) {
     long long c_wait = 0;
     // tiles per lane of a full window: 8 for small records, 4 when a record
     // has more than 2 words (keeps the window's registers in check)
@@ -529,7 +530,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
             const long long cw = clock64();
             __nanosleep(ns);
             c_wait += clock64() - cw;
-            ns = ns < 512 ? 2 * ns : ns;
+            ns = ns < ns_cap ? 2 * ns : ns;
         }
     }
     if (prm.stats != nullptr && lane == 0) {           // debug counters (shared, per warp)

@@ -14,7 +14,7 @@ import workloads  # noqa: E402
 NAMES = ["entry", "ticket", "loaded", "phaseA_sync", "lookback_done", "phaseB_done", "store_read"]
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for name in ["prefix", "tuple2", "order3", "lp1", "hp3"]:
-    for n in [1 << 14, 1 << 18, 1 << 20, 1 << 22]:
+    for n in [3840 * 4, 3840 * 68, 3840 * 273, 3840 * 1092]:
         sig = workloads.BY_NAME[name]
         x = workloads.device_input(n, sig.dtype, 1)
         y = torch.empty_like(x)
