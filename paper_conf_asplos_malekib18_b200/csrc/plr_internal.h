@@ -115,8 +115,14 @@ struct PlanTables {
 };
 
 // small-n kernel geometry: X = 15 elements per thread, W = 8 warps, m = 3840
-constexpr int kSmallX = 15;
-constexpr int kSmallW = 8;
+#ifndef PLR_SMALL_X
+#define PLR_SMALL_X 15
+#endif
+#ifndef PLR_SMALL_W
+#define PLR_SMALL_W 8
+#endif
+constexpr int kSmallX = PLR_SMALL_X;
+constexpr int kSmallW = PLR_SMALL_W;
 // reduce-only kernel geometry (plr_kernels_reduce.cuh): X = 31, W = 8
 // (tile 7936), 3-stage TMA ring, 2 CTAs per SM
 constexpr int kRedX = 31;

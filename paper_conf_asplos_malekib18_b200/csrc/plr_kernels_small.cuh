@@ -62,7 +62,7 @@ struct LayoutS {
 };
 
 template <typename T, typename A, int K, int P, int X, int W, bool REV = false>
-__global__ void __launch_bounds__(W * 32, 2)
+__global__ void __launch_bounds__(W * 32, W >= 16 ? 1 : 2)
 plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = LayoutS<T, A, K, X, W>;
     constexpr int M = L::M;
