@@ -412,7 +412,7 @@ template <typename T, typename A, int K, bool DEC>
 __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, const Tables<T, A>& tb, long long j,
                                                  int lane, uint32_t tagA, uint32_t tagI, A (&Gp)[K],
                                                  const LbStats& lbs, long long c_start = 0, long long c_agg = 0,
-                                                 int ns_cap = 512) {
+                                                 int ns_cap = 512, bool wide_first = false) {
     long long c_wait = 0;
     // tiles per lane of a full window: 8 for small records, 4 when a record
     // has more than 2 words (keeps the window's registers in check)
@@ -430,7 +430,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
 #ifndef PLR_LB_LTPL0
 #define PLR_LB_LTPL0 1
 #endif
-    int ltpl = PLR_LB_LTPL0 < kLogT ? PLR_LB_LTPL0 : kLogT;   // log2 tiles per lane of the first window
+    int ltpl = wide_first ? kLogT : (PLR_LB_LTPL0 < kLogT ? PLR_LB_LTPL0 : kLogT);   // log2 tiles per lane, first window
 #ifndef PLR_LB_NS0
 #define PLR_LB_NS0 32
 #endif

@@ -97,7 +97,38 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 #endif
     const bool resident = (prm.dec_mask & 0x100u) != 0;     // all tiles resident: tile = blockIdx.x
     __shared__ unsigned long long s_tbase;
+    // one TMA bulk load of tile j (+ halo); the ragged tile is loaded by the
+    // compute threads element by element
+    auto issue_load = [&](long long j) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
+        const bool ragged_ = REV ? (j == 0 && n % (unsigned long long)M != 0) : (unsigned long long)(j + 1) * M > n;
+        if (ragged_) return;
+        const uint64_t pol = policy_evict_first();
+        if (REV) {                                   // original tile o, halo after it (zero beyond n)
+            const long long o = ntiles - 1 - j;
+            mbar_arrive_tx(bar, M * sizeof(T));
+            bulk_load(stage, prm.x + (size_t)o * M, M * sizeof(T), bar, pol);
+#pragma unroll
+            for (int q = 0; q < kHalo; q++) {
+                const unsigned long long i = (unsigned long long)(o + 1) * M + q;
+                stage[M + q] = (q < P && i < n) ? prm.x[i] : T(0);
+            }
+        } else if (j == 0) {
+            mbar_arrive_tx(bar, M * sizeof(T));
+            bulk_load(stage + kHalo, prm.x, M * sizeof(T), bar, pol);
+#pragma unroll
+            for (int q = 0; q < kHalo; q++)
+                stage[q] = (q >= kHalo - P && prm.x_hist != nullptr) ? prm.x_hist[q - (kHalo - P)] : T(0);
+        } else {
+            mbar_arrive_tx(bar, (M + kHalo) * sizeof(T));
+            bulk_load(stage, prm.x + (size_t)j * M - kHalo, (M + kHalo) * sizeof(T), bar, pol);
+        }
+    };
     if (tid == 0) {
+        // resident: the tile is known at entry, so its load is issued before
+        // the launch state is read (an L2 round trip, ~0.5 us)
+        if (resident) issue_load((long long)blockIdx.x);
         const unsigned long long tbase = ld_volatile_u64(prm.ticket + 1);
         const uint32_t epoch = (uint32_t)ld_volatile_u64(prm.ticket + 2) + 1u;
         long long j;
@@ -107,6 +138,7 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         } else {
             j = (long long)(atomicAdd(prm.ticket, 1ull) - tbase);
             launch_state_advance(prm.ticket, j, (unsigned long long)ntiles, tbase, epoch);
+            issue_load(j);
         }
 #ifdef PLR_TRACE
         if (prm.stats != nullptr && j == ntiles - 1) prm.stats[9] = t_entry;
@@ -114,31 +146,6 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         PLR_STAMP_LAST(10);
         *s_tile = j;
         s_epoch = epoch;
-        mbar_init(bar, 1);
-        fence_mbar_init();
-        const bool ragged_ = REV ? (j == 0 && n % (unsigned long long)M != 0) : (unsigned long long)(j + 1) * M > n;
-        if (!ragged_) {                              // one TMA bulk load of the tile (+ halo)
-            const uint64_t pol = policy_evict_first();
-            if (REV) {                               // original tile o, halo after it (zero beyond n)
-                const long long o = ntiles - 1 - j;
-#pragma unroll
-                for (int q = 0; q < kHalo; q++) {
-                    const unsigned long long i = (unsigned long long)(o + 1) * M + q;
-                    stage[M + q] = (q < P && i < n) ? prm.x[i] : T(0);
-                }
-                mbar_arrive_tx(bar, M * sizeof(T));
-                bulk_load(stage, prm.x + (size_t)o * M, M * sizeof(T), bar, pol);
-            } else if (j == 0) {
-#pragma unroll
-                for (int q = 0; q < kHalo; q++)
-                    stage[q] = (q >= kHalo - P && prm.x_hist != nullptr) ? prm.x_hist[q - (kHalo - P)] : T(0);
-                mbar_arrive_tx(bar, M * sizeof(T));
-                bulk_load(stage + kHalo, prm.x, M * sizeof(T), bar, pol);
-            } else {
-                mbar_arrive_tx(bar, (M + kHalo) * sizeof(T));
-                bulk_load(stage, prm.x + (size_t)j * M - kHalo, (M + kHalo) * sizeof(T), bar, pol);
-            }
-        }
     }
     __syncthreads();
     const long long j = *s_tile;
@@ -273,8 +280,9 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             const LbStats lbs{s_lbst};
             lbs.init(lane);
             __syncwarp();
-            // every predecessor publishes at about the same time: short, flat sleeps
-            lookback_generic<T, A, K, DECF>(prm, tb, j, lane, tagA, tagI, Gp, lbs, 0, 0, 64);
+            // every predecessor publishes at about the same time: the widest
+            // window from the start, short flat sleeps
+            lookback_generic<T, A, K, DECF>(prm, tb, j, lane, tagA, tagI, Gp, lbs, 0, 0, 64, true);
             __syncwarp();
             lbs.flush(prm.stats, lane);
         }

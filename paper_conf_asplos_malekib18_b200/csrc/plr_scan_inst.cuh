@@ -61,8 +61,9 @@ namespace inst {
 #define PLR_GEN_TMEM (PLR_GEN_KIND != 0)
 // re-read kernel (measured r01r-r01u): X = 31, W = 8 (tile 7936), 3 look-back
 // warps, 2 HBM load stages, 5 L2 re-read / store stages, phase-B lag 8 tiles,
-// look-back units of 4 tiles (G >= 5 hung at NS = 9 before the chained agg
-// waits of DESIGN.md §10)
+// look-back units of 6 tiles with NS = 10 slots (r03d, profiles/r03d_rr_unit_cmp.txt:
+// tuple3 0.910 -> 0.923, order2 0.936 -> 0.944 against G = 4 / NS = 9; the
+// configuration hung before the chained agg waits of DESIGN.md §10)
 #ifndef PLR_RR_X
 #define PLR_RR_X 31
 #endif
@@ -79,10 +80,10 @@ namespace inst {
 #define PLR_RR_SB 5         // phase-B (L2 re-read + y store) stages
 #endif
 #ifndef PLR_RR_NS
-#define PLR_RR_NS 9         // slots: phase B lags phase A by NS-1 tiles (L2 reuse distance)
+#define PLR_RR_NS 10        // slots: phase B lags phase A by NS-1 tiles (L2 reuse distance)
 #endif
 #ifndef PLR_RR_G
-#define PLR_RR_G 4          // tiles per look-back unit (one ticket, one look-back)
+#define PLR_RR_G 6          // tiles per look-back unit (one ticket, one look-back)
 #endif
 #ifndef PLR_TM_X
 #define PLR_TM_X 15

@@ -20,15 +20,21 @@ for name in ["prefix", "tuple2", "order3", "lp1", "hp3"]:
         y = torch.empty_like(x)
         plan = plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
         rows = []
+        lb = []
         for r in range(7):
             flush.fill_(r)
             torch.cuda.synchronize()
             plan(x, y)
             torch.cuda.synchronize()
-            t = plan.debug_stats(reset=True)["trace"]
+            st = plan.debug_stats(reset=True)
+            t = st["trace"]
             if r >= 2:
                 rows.append([(v - t[0]) if v else -1 for v in t])
+                lb.append(st)
         med = [sorted(c)[len(c) // 2] for c in zip(*rows)]
-        print(json.dumps({"sig": name, "n": n, "tiles": -(-n // plan.info["tile_elems"]) if False else None,
-                          "ns_after_entry": dict(zip(NAMES, med))}), flush=True)
+        nl = max(1, sum(s["lookbacks"] for s in lb))
+        per = {k: round(sum(s[k] for s in lb) / nl, 2) for k in ("windows", "waits", "depth_sum", "cyc_lookback",
+                                                                  "cyc_sleep", "cyc_load", "cyc_fold")}
+        print(json.dumps({"sig": name, "n": n, "ns_after_entry": dict(zip(NAMES, med)),
+                          "per_lookback_mean": per}), flush=True)
         plan.close()
