@@ -101,7 +101,8 @@ typedef struct {
                                   kernel parameters                                   */
     int tiles_per_unit;        /* G: consecutive tiles per ticket / status record / look-back */
     int kernel_kind;           /* scan kernel: 0 DECAY single-hop pipeline, 1 TMEM-parking,
-                                  2 L2 re-read (generic classes), 3 generic smem pipeline */
+                                  2 L2 re-read (generic classes), 3 generic smem pipeline,
+                                  4 DECAY single-hop with TMEM-parked map outputs        */
     int acc_bits;              /* accumulation of the chunk recurrence and carries: 32 (the
                                   data type) or 64 (fp64, reading R16)       */
     double cond_bound;         /* float: the planner's a-priori error bound of fp32

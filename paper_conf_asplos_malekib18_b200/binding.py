@@ -185,7 +185,8 @@ class Plan:
             pass
 
     KERNEL_NAMES = {0: "plr_scan_kernel (DECAY single-hop pipeline)", 1: "plr_scan_tmem_kernel (TMEM parking)",
-                    2: "plr_scan_rr_kernel (L2 re-read)", 3: "plr_scan_kernel (generic pipeline)"}
+                    2: "plr_scan_rr_kernel (L2 re-read)", 3: "plr_scan_kernel (generic pipeline)",
+                    4: "plr_scan_dect_kernel (DECAY, map outputs parked in TMEM)"}
 
     def kernel_name(self) -> str:
         return self.KERNEL_NAMES.get(self.info["kernel_kind"], "?")

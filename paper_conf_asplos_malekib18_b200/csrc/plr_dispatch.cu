@@ -18,7 +18,7 @@ Geometry class_geometry(bool decay, int k, bool acc64) {
 int scan_stages(const PlanTables& pt) { return pt.geo.S; }
 
 int kernel_kind(const PlanTables& pt) {
-    if (pt.decay_flag) return 0;
+    if (pt.decay_flag) return (pt.acc64 ? inst::CfgDec64::DT : inst::CfgDec::DT) ? 4 : 0;
     const int kind = inst::gen_kind(pt.k);
     return kind == 0 ? 3 : kind;
 }

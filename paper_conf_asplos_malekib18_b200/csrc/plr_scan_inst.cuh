@@ -5,6 +5,7 @@
 #include "plr_kernels.cuh"
 #include "plr_kernels_tmem.cuh"
 #include "plr_kernels_rr.cuh"
+#include "plr_kernels_dect.cuh"
 #include "plr_launch.h"
 #include <atomic>
 #include <type_traits>
@@ -113,11 +114,29 @@ constexpr int gen_kind(int k) { return k == 1 ? PLR_K1_KIND : PLR_GEN_KIND; }
 // U1_: look-back units of one tile (the small-n launches, plr_api.cu), else
 // PLR_RR_G / PLR_TM_G tiles per unit
 // SEED_: phase B runs the seeded serial recurrence (plr_scan_kernel SEED)
-template <int S_, int D_, int NL_, int X_, int W_, int MINB_, bool DEC_, bool U1_ = false, bool SEED_ = false>
+// DT_: the forward DECAY pass runs plr_scan_dect_kernel (map outputs parked
+// in TMEM, split load / store rings: PLR_DT_SL / PLR_DT_ST stages, lag PLR_DT_D)
+template <int S_, int D_, int NL_, int X_, int W_, int MINB_, bool DEC_, bool U1_ = false, bool SEED_ = false,
+          bool DT_ = false>
 struct Cfg {
     static constexpr int S = S_, D = D_, NL = NL_, X = X_, W = W_, MINB = MINB_;
-    static constexpr bool DEC = DEC_, U1 = U1_, SEED = SEED_;
+    static constexpr bool DEC = DEC_, U1 = U1_, SEED = SEED_, DT = DT_;
 };
+#ifndef PLR_DT_SL
+#define PLR_DT_SL 2
+#endif
+#ifndef PLR_DT_ST
+#define PLR_DT_ST 2
+#endif
+#ifndef PLR_DT_D
+#define PLR_DT_D 1
+#endif
+#ifndef PLR_DEC_DT
+#define PLR_DEC_DT 0
+#endif
+#ifndef PLR_DEC64_DT
+#define PLR_DEC64_DT 1
+#endif
 // DECAY phase B (measured r03b at 2^30, fraction of copy): fp32 plans keep
 // the correction y = l + sum_r S_r h^(r)_u (independent FMAs; seeded: LP1
 // 0.99 -> 0.95, HP2 0.98 -> 0.95, the serial chain is exposed); fp64-
@@ -130,9 +149,10 @@ struct Cfg {
 #ifndef PLR_DEC64_SEED
 #define PLR_DEC64_SEED 1
 #endif
-using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true, false, PLR_DEC_SEED>;
+using CfgDec = Cfg<PLR_DEC_S, PLR_DEC_D, PLR_DEC_NL, PLR_DEC_X, PLR_DEC_W, PLR_DEC_MINB, true, false, PLR_DEC_SEED,
+                   PLR_DEC_DT != 0>;
 using CfgDec64 = Cfg<PLR_DEC64_S, PLR_DEC64_D, PLR_DEC64_NL, PLR_DEC64_X, PLR_DEC64_W, PLR_DEC64_MINB, true, false,
-                     PLR_DEC64_SEED>;
+                     PLR_DEC64_SEED, PLR_DEC64_DT != 0>;
 using CfgGen = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false>;
 using CfgGen1 = Cfg<PLR_GEN_S, PLR_GEN_D, PLR_GEN_NL, PLR_GEN_X, PLR_GEN_W, PLR_GEN_MINB, false, true>;
 
@@ -171,6 +191,13 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
             if (la.reverse)
                 kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB, C::SEED,
                                              true>;
+        }
+        if constexpr (C::DEC && STORE && C::DT) {         // forward DECAY pass with TMEM-parked map outputs
+            if (!la.reverse) {
+                kern = &dev::plr_scan_dect_kernel<T, A, K, P, C::X, C::W, PLR_DT_SL, PLR_DT_ST, PLR_DT_D, C::MINB>;
+                smem = dev::LayoutDT<T, A, K, C::X, C::W, PLR_DT_SL, PLR_DT_ST, PLR_DT_D + 1>::bytes;
+                threads = (C::W + 2) * 32;
+            }
         }
         smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
         threads = (C::W + 1 + C::NL) * 32;
