@@ -87,11 +87,16 @@ static uint64_t unit1_waves() {
 }
 
 // Sizes up to this many elements run the small-n kernel (one CTA per tile,
-// no pipeline, profiles/*_sweep.md); PLR_SMALL_MAX
+// no pipeline).  Measured crossover against the
+// persistent kernels (profiles/r03e_sweep_auto.md vs r03c_sweep_big.md):
+// 2^21 for DECAY and first-order plans (single-hop / scalar look-back), 2^17
+// for k >= 2 non-decaying plans (their look-back over every predecessor
+// costs more than the persistent kernels' units beyond that).  PLR_SMALL_MAX
 // overrides it at plan creation (0: never).
-static size_t small_max_default() {
+static size_t small_max_default(const PlanTables& pt) {
     const char* e = std::getenv("PLR_SMALL_MAX");
-    return e != nullptr ? (size_t)std::strtoull(e, nullptr, 10) : ((size_t)1 << 22);
+    if (e != nullptr) return (size_t)std::strtoull(e, nullptr, 10);
+    return (pt.decay_flag || pt.k == 1) ? ((size_t)1 << 21) : ((size_t)1 << 17);
 }
 
 // ============================================================ helpers =====
@@ -441,13 +446,16 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
             if ((e = cudaMalloc(&plan->d_rd, rb)) != cudaSuccess) return bail(e, "alloc reduce records");
         }
     }
-    plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default()) : 0;
+    plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default(plan->pt)) : 0;
     plan->small_ctas = small_ctas;
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
-    // status slots cover the small-n tiles up to n_max: the anticausal pass of
-    // a non-DECAY plan runs the small-n kernel at every size
-    plan->max_tiles = std::max<uint64_t>(plan->max_tiles, (n_max + ms - 1) / ms);
+    // status slots cover the small-n tiles up to small_max -- up to n_max for
+    // non-DECAY plans, whose anticausal pass runs the small-n kernel at every
+    // size.  (Sizing the DECAY plans' slots for n_max small tiles too doubled
+    // the array and cost their forward pass ~3 % at 2^30, r03e A/B.)
+    const size_t small_cover = plan->pt.decay_flag ? plan->small_max : n_max;
+    plan->max_tiles = std::max<uint64_t>(plan->max_tiles, (small_cover + ms - 1) / ms);
     if (plan->max_tiles > (1ull << 31)) { plr_plan_destroy(plan); return fail(PLR_ERR_SIZE, "n_max too large"); }
     plan->status_slots = 1;
     while (plan->status_slots < plan->max_tiles) plan->status_slots <<= 1;
