@@ -187,6 +187,8 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
         threads = (TC::W + 1 + TC::NL) * 32;
     } else {
         kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB, C::SEED>;
+        smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
+        threads = (C::W + 1 + C::NL) * 32;
         if constexpr (C::DEC && STORE) {                 // the anticausal pass (DECAY plans)
             if (la.reverse)
                 kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB, C::SEED,
@@ -199,8 +201,6 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
                 threads = (C::W + 2) * 32;
             }
         }
-        smem = dev::Layout<T, A, K, C::X, C::W, C::S, C::D>::bytes;
-        threads = (C::W + 1 + C::NL) * 32;
     }
     // the > 48 KB dynamic shared memory opt-in is a per-device (context)
     // attribute: one bit per device and kernel, set once (racing sets are
