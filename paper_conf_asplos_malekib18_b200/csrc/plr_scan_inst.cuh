@@ -29,13 +29,20 @@ namespace inst {
 #define PLR_DEC_W 8
 #define PLR_DEC_MINB 2
 #endif
+// fp64-accumulation DECAY (LP3, HP3): the TMEM-parked kernel
+// (plr_scan_dect_kernel); a kernel that allocates TMEM runs one CTA per SM
+// (profiles/r03g_tmem_occupancy.txt), so one wide CTA: X = 23, W = 16
+// (tile 11776), 2 load + 2 store stages (measured r03h: LP3 0.89, HP3 0.87
+// of a copy, against 0.83 / 0.81 for the in-place kernel at 3 CTAs/SM with
+// X = 31, W = 4).  The anticausal pass runs the in-place kernel with the
+// same geometry (the plan's tables are built for one geometry).
 #ifndef PLR_DEC64_S
 #define PLR_DEC64_S 4
 #define PLR_DEC64_D 1
 #define PLR_DEC64_NL 1
-#define PLR_DEC64_X 31
-#define PLR_DEC64_W 4
-#define PLR_DEC64_MINB 3
+#define PLR_DEC64_X 23
+#define PLR_DEC64_W 16
+#define PLR_DEC64_MINB 1
 #endif
 #ifndef PLR_GEN_S
 #define PLR_GEN_S 3
