@@ -31,16 +31,16 @@ namespace inst {
 #endif
 // fp64-accumulation DECAY (LP3, HP3): the TMEM-parked kernel
 // (plr_scan_dect_kernel); a kernel that allocates TMEM runs one CTA per SM
-// (profiles/r03g_tmem_occupancy.txt), so one wide CTA: X = 23, W = 16
-// (tile 11776), 2 load + 2 store stages (measured r03h: LP3 0.89, HP3 0.87
+// (profiles/r03g_tmem_occupancy.txt), so one wide CTA: X = 27, W = 16
+// (tile 13824), 2 load + 2 store stages (measured r03i: LP3 0.94, HP3 0.94
 // of a copy, against 0.83 / 0.81 for the in-place kernel at 3 CTAs/SM with
-// X = 31, W = 4).  The anticausal pass runs the in-place kernel with the
+// X = 31, W = 4; profiles/r03h_dect_geometry_cmp.txt, r03i_*).  The anticausal pass runs the in-place kernel with the
 // same geometry (the plan's tables are built for one geometry).
 #ifndef PLR_DEC64_S
 #define PLR_DEC64_S 4
 #define PLR_DEC64_D 1
 #define PLR_DEC64_NL 1
-#define PLR_DEC64_X 23
+#define PLR_DEC64_X 27
 #define PLR_DEC64_W 16
 #define PLR_DEC64_MINB 1
 #endif
