@@ -41,7 +41,9 @@ struct plr_plan {
     int ctas_per_sm = 0;
     size_t n_max = 0;
     uint64_t max_tiles = 0;
-    uint64_t status_slots = 0;              // power of two >= max_tiles
+    uint64_t status_slots = 0;              // power of two >= max_tiles (persistent kernels' tiles)
+    uint64_t status_slots_s = 0;            // the small-n kernel's own status array (its tiles)
+    unsigned long long* d_status_s = nullptr;
     unsigned long long* d_ticket = nullptr;
     unsigned long long* d_status = nullptr;
     uint32_t epoch = 0;                 // host count of launches since the last reset (overflow guard)
@@ -247,20 +249,23 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     if (n > plan->n_max) return fail(PLR_ERR_SIZE, "n exceeds the plan's n_max");
     if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
         CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, stream), "status reset");
+        CUDA_TRY(cudaMemsetAsync(plan->d_status_s, 0, plan->status_slots_s * kStatusMaxBytes, stream), "status reset");
         CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, kTicketBytes, stream), "ticket reset");
         plan->epoch = 0;
         plan->dirty = false;
     }
     // small n: one CTA per tile, no pipeline; the anticausal pass of a
-    // non-DECAY plan runs the small-n kernel at every size
-    if (n <= plan->small_max || (reverse && !plan->pt.decay_flag)) {
+    // non-DECAY or fp64-accumulation plan runs the small-n kernel at every
+    // size (the in-place DECAY kernel's fp64 footprint at the wide geometry
+    // exceeds shared memory)
+    if (n <= plan->small_max || (reverse && (!plan->pt.decay_flag || plan->pt.acc64))) {
         const uint64_t ms = (uint64_t)plan->pt.geo_s.tile();
         plan->epoch++;
         LaunchArgs la;
         la.x = x; la.y = store ? y : nullptr; la.n = n; la.ntiles = (n + ms - 1) / ms;
         la.ticket = plan->d_ticket;
-        la.status = plan->d_status;
-        la.status_mask = plan->status_slots - 1;
+        la.status = plan->d_status_s;
+        la.status_mask = plan->status_slots_s - 1;
         la.decay = plan->pt.decay_s;
         la.dec_mask = plan->pt.dec_mask_s;
         // every tile resident at once (one wave): tile index = blockIdx.x, no
@@ -360,6 +365,7 @@ plr_status plr_plan_destroy(plr_plan* plan) {
     if (plan == nullptr) return PLR_OK;
     cudaFree(plan->d_ticket);
     cudaFree(plan->d_status);
+    cudaFree(plan->d_status_s);
     cudaFree(plan->d_lane);
     cudaFree(plan->d_lane_s);
     cudaFree(plan->d_rd);
@@ -450,19 +456,27 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     plan->small_ctas = small_ctas;
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
-    // status slots cover the small-n tiles up to small_max -- up to n_max for
-    // non-DECAY plans, whose anticausal pass runs the small-n kernel at every
-    // size.  (Sizing the DECAY plans' slots for n_max small tiles too doubled
-    // the array and cost their forward pass ~3 % at 2^30, r03e A/B.)
-    const size_t small_cover = plan->pt.decay_flag ? plan->small_max : n_max;
-    plan->max_tiles = std::max<uint64_t>(plan->max_tiles, (small_cover + ms - 1) / ms);
-    if (plan->max_tiles > (1ull << 31)) { plr_plan_destroy(plan); return fail(PLR_ERR_SIZE, "n_max too large"); }
+    // Two status arrays: the persistent kernels' (their tiles up to n_max)
+    // and the small-n kernel's (its tiles up to small_max -- up to n_max for
+    // plans whose anticausal pass runs the small-n kernel at every size).
+    // One shared array sized for the small tiles doubled the persistent
+    // kernels' and cost their forward pass ~3 % at 2^30 (r03e/r03f A/B).
+    const bool rev_small = !plan->pt.decay_flag || plan->pt.acc64;
+    const uint64_t small_tiles = std::max<uint64_t>(1, ((rev_small ? n_max : plan->small_max) + ms - 1) / ms);
+    if (plan->max_tiles > (1ull << 31) || small_tiles > (1ull << 31)) {
+        plr_plan_destroy(plan);
+        return fail(PLR_ERR_SIZE, "n_max too large");
+    }
     plan->status_slots = 1;
     while (plan->status_slots < plan->max_tiles) plan->status_slots <<= 1;
+    plan->status_slots_s = 1;
+    while (plan->status_slots_s < small_tiles) plan->status_slots_s <<= 1;
     if ((e = cudaMalloc(&plan->d_ticket, kTicketBytes)) != cudaSuccess) return bail(e, "alloc ticket");
     if ((e = cudaMalloc(&plan->d_status, plan->status_slots * kStatusMaxBytes)) != cudaSuccess) return bail(e, "alloc status");
+    if ((e = cudaMalloc(&plan->d_status_s, plan->status_slots_s * kStatusMaxBytes)) != cudaSuccess) return bail(e, "alloc status");
     if ((e = cudaMemset(plan->d_ticket, 0, kTicketBytes)) != cudaSuccess) return bail(e, "memset");
     if ((e = cudaMemset(plan->d_status, 0, plan->status_slots * kStatusMaxBytes)) != cudaSuccess) return bail(e, "memset");
+    if ((e = cudaMemset(plan->d_status_s, 0, plan->status_slots_s * kStatusMaxBytes)) != cudaSuccess) return bail(e, "memset");
     const bool acc64 = dtype == PLR_FLOAT32 && plan->pt.acc64;
     const size_t lane_bytes = (size_t)k * k * 32 * (acc64 ? 8 : 4);
     if ((e = cudaMalloc(&plan->d_lane, lane_bytes)) != cudaSuccess) return bail(e, "alloc lane table");
@@ -566,7 +580,7 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->decay_len = plan->pt.decay_len;
     info->fixup_len = plan->pt.fixup_len;
     info->n_max = plan->n_max;
-    info->scratch_bytes = 8 + plan->status_slots * kStatusMaxBytes + (size_t)plan->pt.k * plan->pt.k * 128 +
+    info->scratch_bytes = 8 + (plan->status_slots + plan->status_slots_s) * kStatusMaxBytes + (size_t)plan->pt.k * plan->pt.k * 128 +
                           (size_t)plan->pt.fixup_len * kAug * 4 + 64;
     info->ctas_per_sm = plan->ctas_per_sm;
     info->num_sms = plan->num_sms;
@@ -674,6 +688,7 @@ plr_status plr_reduce(plr_plan* plan, const void* x, size_t n, void* payload, vo
             // contiguous-range streaming fold, no look-back (plr_kernels_reduce.cuh)
             if (plan->dirty || plan->epoch >= 0x7ffffff0u) {
                 CUDA_TRY(cudaMemsetAsync(plan->d_status, 0, plan->status_slots * kStatusMaxBytes, s), "status reset");
+                CUDA_TRY(cudaMemsetAsync(plan->d_status_s, 0, plan->status_slots_s * kStatusMaxBytes, s), "status reset");
                 CUDA_TRY(cudaMemsetAsync(plan->d_ticket, 0, kTicketBytes, s), "ticket reset");
                 plan->epoch = 0;
                 plan->dirty = false;

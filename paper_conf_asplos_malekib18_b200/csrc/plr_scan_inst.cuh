@@ -14,33 +14,29 @@ namespace plr {
 namespace inst {
 
 // Pipeline configs (measured on B200):
-//   DECAY (single-hop look-back): shallow pipeline, 3 CTAs/SM fit:
-//     S = 4 stages, phase-A lead D = 1, one look-back warp;
-//   generic (multi-tile look-back): deep pipeline so predecessors' aggregates
-//     are published before a tile looks back: S = 6, D = 3, two look-back warps.
-//   fp32 DECAY: X = 23, W = 8 (tile 5888), 2 CTAs/SM; fp64-accumulation
-//   DECAY (issue-bound, R16): X = 31, W = 4 (tile 3968), 3 CTAs/SM, so the
-//   per-thread scan overhead is amortised over more elements (measured r01q).
+//   DECAY, fp32 and fp64 accumulation: the forward pass runs the
+//   TMEM-parked kernel (plr_scan_dect_kernel); a kernel that allocates TMEM
+//   runs one CTA per SM (profiles/r03g_tmem_occupancy.txt), so one wide CTA:
+//   X = 31, W = 16 (tile 15872), 2 load stages + 1 store stage (measured
+//   r03k: LP3 1.01, HP3 0.995 of a copy, against 0.83 / 0.81 for the
+//   in-place kernel at 3 CTAs/SM with X = 31, W = 4; the fp32 rows 1.04
+//   against 0.97-1.01 in place; profiles/r03h_*, r03i_*, r03k_*).  The
+//   in-place kernel (S = 3 stages at this geometry) serves the anticausal
+//   pass of fp32 plans; fp64 plans run that on the small-n kernel.
+//   generic (multi-tile look-back, GEN_KIND 0, not shipped): S = 3, D = 1.
 #ifndef PLR_DEC_S
-#define PLR_DEC_S 4
+#define PLR_DEC_S 3
 #define PLR_DEC_D 1
 #define PLR_DEC_NL 1
-#define PLR_DEC_X 23
-#define PLR_DEC_W 8
-#define PLR_DEC_MINB 2
+#define PLR_DEC_X 31
+#define PLR_DEC_W 16
+#define PLR_DEC_MINB 1
 #endif
-// fp64-accumulation DECAY (LP3, HP3): the TMEM-parked kernel
-// (plr_scan_dect_kernel); a kernel that allocates TMEM runs one CTA per SM
-// (profiles/r03g_tmem_occupancy.txt), so one wide CTA: X = 27, W = 16
-// (tile 13824), 2 load + 2 store stages (measured r03i: LP3 0.94, HP3 0.94
-// of a copy, against 0.83 / 0.81 for the in-place kernel at 3 CTAs/SM with
-// X = 31, W = 4; profiles/r03h_dect_geometry_cmp.txt, r03i_*).  The anticausal pass runs the in-place kernel with the
-// same geometry (the plan's tables are built for one geometry).
 #ifndef PLR_DEC64_S
-#define PLR_DEC64_S 4
+#define PLR_DEC64_S 3
 #define PLR_DEC64_D 1
 #define PLR_DEC64_NL 1
-#define PLR_DEC64_X 27
+#define PLR_DEC64_X 31
 #define PLR_DEC64_W 16
 #define PLR_DEC64_MINB 1
 #endif
@@ -133,13 +129,13 @@ struct Cfg {
 #define PLR_DT_SL 2
 #endif
 #ifndef PLR_DT_ST
-#define PLR_DT_ST 2
+#define PLR_DT_ST 1
 #endif
 #ifndef PLR_DT_D
 #define PLR_DT_D 1
 #endif
 #ifndef PLR_DEC_DT
-#define PLR_DEC_DT 0
+#define PLR_DEC_DT 1
 #endif
 #ifndef PLR_DEC64_DT
 #define PLR_DEC64_DT 1
