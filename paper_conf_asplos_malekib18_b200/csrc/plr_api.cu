@@ -703,7 +703,8 @@ plr_status plr_reduce(plr_plan* plan, const void* x, size_t n, void* payload, vo
             la.decay = 0;
             la.x_hist = nullptr; la.y_hist = nullptr; la.y_tail = y_tail;
             la.lane_T = nullptr;
-            la.grid = (int)std::min<uint64_t>(la.ntiles, (uint64_t)plan->num_sms * plan->reduce_ctas);
+            la.grid = (int)std::min<uint64_t>(std::min<uint64_t>(la.ntiles, (uint64_t)plan->num_sms * plan->reduce_ctas),
+                                                 (uint64_t)kRedMaxGrid);
             la.store = false;
             la.stream = s;
             cudaError_t e = launch_reduce(plan->pt, la);

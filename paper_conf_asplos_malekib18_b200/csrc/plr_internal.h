@@ -128,6 +128,7 @@ constexpr int kSmallW = PLR_SMALL_W;
 constexpr int kRedX = 31;
 constexpr int kRedW = 8;
 constexpr int kRedS = 3;
+constexpr int kRedMaxGrid = 1024;   // reduce-only grid cap (the last CTA copies every CTA record to smem)
 
 // planner (host, plr_planner.cpp)
 plr_status plan_tables(const double* a, int p, const double* b, int k, plr_dtype dtype,

@@ -242,22 +242,36 @@ plr_reduce_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         }
     }
     __syncthreads();
-    // the last CTA folds the records in order: E = T(L_c) E + acc_c
-    if (*s_last && tid == 0) {
-        __threadfence();
+    // the last CTA folds the records in order: E = T(L_c) E + acc_c.  Every
+    // thread first copies records tid, tid + blockDim, ... into the (now idle)
+    // stage ring, so the grid's records cost one L2 round trip, not one per
+    // record (a serial chain of dependent loads was ~0.3 us x grid)
+    if (!*s_last) return;
+    constexpr int RW = kMaxK;                                     // values per copied record
+    static_assert(L::off_wagg >= (size_t)kRedMaxGrid * (8 + RW * sizeof(A)), "record copy fits the stage ring");
+    unsigned long long* slen = reinterpret_cast<unsigned long long*>(smem + L::off_stage);
+    A* srec = reinterpret_cast<A*>(slen + grid);
+    __threadfence();
+    for (int c = tid; c < grid; c += (int)blockDim.x) {
+        const volatile unsigned long long* rec = rd_record<A>(prm.status, c);
+        const volatile A* ra = reinterpret_cast<const volatile A*>(rec);
+        slen[c] = rec[(kStatusMaxBytes / 8) - 1];
+#pragma unroll
+        for (int e = 0; e < K; e++) srec[(size_t)c * RW + e] = ra[e];
+    }
+    __syncthreads();
+    if (tid == 0) {
         A E[K];
 #pragma unroll
         for (int e = 0; e < K; e++) E[e] = A(0);
         A Tq[kMaxK * kMaxK];
         companion_pow<A, K>(tb.c, (unsigned long long)q * M, Tq);
         for (int c = 0; c < grid; c++) {
-            const volatile unsigned long long* rec = rd_record<A>(prm.status, c);
-            const unsigned long long len = rec[(kStatusMaxBytes / 8) - 1];
+            const unsigned long long len = slen[c];
             if (len == 0) continue;
             A a_[K];
-            const volatile A* ra = reinterpret_cast<const volatile A*>(rec);
 #pragma unroll
-            for (int e = 0; e < K; e++) a_[e] = ra[e];
+            for (int e = 0; e < K; e++) a_[e] = srec[(size_t)c * RW + e];
             if (len == (unsigned long long)q * M) {
                 matvec_acc<A, K>(a_, Tq, E);
             } else {
