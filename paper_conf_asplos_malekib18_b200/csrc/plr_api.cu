@@ -51,6 +51,7 @@ struct plr_plan {
     void* d_lane_s = nullptr;           // lane table T(X_s l) of the small-n kernel
     size_t small_max = 0;               // n <= small_max: the small-n kernel (plr_kernels_small.cuh)
     int small_ctas = 0;                 // its CTAs per SM (all tiles resident: tile = blockIdx.x)
+    int small_clusters = 0;             // co-resident clusters of kSmallC small-n CTAs (0: no cluster launches)
     int reduce_ctas = 0;                // CTAs per SM of the reduce-only kernel (0: not available)
     unsigned long long* d_rd = nullptr; // its per-CTA records (kStatusMaxBytes each)
     void* d_scan_tmp = nullptr;         // CUB temp storage of the Scan comparator
@@ -275,6 +276,15 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
             return e == nullptr || e[0] != '0';
         }();
         if (resident_ok && la.ntiles <= (uint64_t)plan->num_sms * plan->small_ctas) la.dec_mask |= 0x100u;
+        // non-decaying forward launches of several tiles whose clusters are
+        // all co-resident: the cluster look-back (PLR_SMALL_CLUSTER=0 turns it off)
+        const char* ce = std::getenv("PLR_SMALL_CLUSTER");
+        const bool cluster_ok = ce == nullptr || ce[0] != '0';
+        if (cluster_ok && resident_ok && !reverse && !plan->pt.decay_s && la.ntiles >= 2 &&
+            (la.ntiles + kSmallC - 1) / kSmallC <= (uint64_t)plan->small_clusters) {
+            la.cluster = true;
+            la.dec_mask |= 0x100u;
+        }
         la.x_hist = x_hist; la.y_hist = y_hist; la.y_tail = y_tail;
         la.lane_T = plan->d_lane_s;
         la.stats = plan->d_stats;
@@ -454,6 +464,12 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     }
     plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default(plan->pt)) : 0;
     plan->small_ctas = small_ctas;
+    if (!plan->pt.decay_s && small_ctas >= 1) {
+        if ((e = small_cluster_occupancy(plan->pt, &plan->small_clusters)) != cudaSuccess) {
+            (void)cudaGetLastError();                          // no cluster launches on this device
+            plan->small_clusters = 0;
+        }
+    }
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
     // Two status arrays: the persistent kernels' (their tiles up to n_max)

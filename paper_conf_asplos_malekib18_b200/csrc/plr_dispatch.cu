@@ -58,6 +58,14 @@ cudaError_t small_occupancy(const PlanTables& pt, int* ctas_per_sm) {
     return launch_small(pt, la);
 }
 
+cudaError_t small_cluster_occupancy(const PlanTables& pt, int* clusters) {
+    LaunchArgs la{};
+    la.occupancy_out = clusters;
+    la.cluster = true;
+    la.ntiles = 1;
+    return launch_small(pt, la);
+}
+
 cudaError_t scan_occupancy(const PlanTables& pt, int* ctas_per_sm) {
     LaunchArgs la{};
     la.store = true;

@@ -123,6 +123,13 @@ struct PlanTables {
 #endif
 constexpr int kSmallX = PLR_SMALL_X;
 constexpr int kSmallW = PLR_SMALL_W;
+// small-n cluster launches (non-decaying, forward, every tile resident):
+// clusters of kSmallC tiles exchange aggregates over DSMEM, the look-back
+// runs over cluster records (plr_kernels_small.cuh)
+#ifndef PLR_SMALL_C
+#define PLR_SMALL_C 8
+#endif
+constexpr int kSmallC = PLR_SMALL_C;
 // reduce-only kernel geometry (plr_kernels_reduce.cuh): X = 31, W = 8
 // (tile 7936), 3-stage TMA ring, 2 CTAs per SM
 constexpr int kRedX = 31;

@@ -407,8 +407,11 @@ struct LbStats {
 // tiles and the inclusive carry of the first "I" tile.  Each poll reads a
 // lane-interleaved window (all loads in flight together), folds its ready
 // prefix (up to the first not-ready or first inclusive tile) and never
-// re-reads folded tiles.  Called by one full warp.
-template <typename T, typename A, int K, bool DEC>
+// re-reads folded tiles.  Called by one full warp.  LOGU: the records are
+// those of units of 2^LOGU table units (T(2^LOGU U 2^s) = Tpow[s + LOGU]; the
+// small-n cluster kernel's cluster records), valid while a look-back folds
+// fewer than 2^(9 - LOGU) records.
+template <typename T, typename A, int K, bool DEC, int LOGU = 0>
 __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, const Tables<T, A>& tb, long long j,
                                                  int lane, uint32_t tagA, uint32_t tagI, A (&Gp)[K],
                                                  const LbStats& lbs, long long c_start = 0, long long c_agg = 0,
@@ -483,7 +486,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
                     A nr[K];
 #pragma unroll
                     for (int q = 0; q < K; q++) nr[q] = v[t][q];
-                    matvec_acc<A, K>(nr, tb.Tpow[5], r);           // T(32 m)
+                    matvec_acc<A, K>(nr, tb.Tpow[5 + LOGU], r);    // T(32 m)
 #pragma unroll
                     for (int q = 0; q < K; q++) r[q] = nr[q];
                 }
@@ -494,7 +497,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
                 A o2[K];
 #pragma unroll
                 for (int q = 0; q < K; q++) o2[q] = shfl_down(r[q], 1 << s2);
-                matvec_acc<A, K>(r, tb.Tpow[s2], o2);
+                matvec_acc<A, K>(r, tb.Tpow[s2 + LOGU], o2);
             }
             A R[K];
 #pragma unroll
@@ -505,7 +508,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
             // skip the folded tiles: Tacc *= T(e m) (binary powers; unrolled so
             // compile-time tables fold)
 #pragma unroll
-            for (int s2 = 0; s2 < 9; s2++) {
+            for (int s2 = 0; s2 + LOGU < 9; s2++) {
                 if (!((e >> s2) & 1)) continue;
                 A nt[K * kMaxK];
 #pragma unroll
@@ -514,7 +517,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
                     for (int c2 = 0; c2 < K; c2++) {
                         A a2 = A(0);
 #pragma unroll
-                        for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], tb.Tpow[s2][t * kMaxK + c2], a2);
+                        for (int t = 0; t < K; t++) a2 = mad(Tacc[q * kMaxK + t], tb.Tpow[s2 + LOGU][t * kMaxK + c2], a2);
                         nt[q * kMaxK + c2] = a2;
                     }
 #pragma unroll

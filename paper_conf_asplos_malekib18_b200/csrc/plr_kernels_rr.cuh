@@ -222,8 +222,18 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         } else if (lane == 2) {                                     // storer
             // every stage goes back to loader B as soon as its bulk store has
             // read it (the stage is the next re-load's destination)
+            // PLR_RR_STQ bulk stores in flight: the stage of position t goes
+            // back once the store of position t + STQ - 1 is issued and every
+            // older store has read its stage (one bulk group per position,
+            // empty for a ragged or unstored tile)
+#ifndef PLR_RR_STQ
+#define PLR_RR_STQ 1
+#endif
+            constexpr int STQ = PLR_RR_STQ;
+            static_assert(STQ >= 1 && STQ <= SB && STQ <= 4, "stores in flight");
             const uint64_t pol = policy_evict_first();
-            for (int t = 0;; t++) {
+            int t = 0;
+            for (;; t++) {
                 const int sb = t % SB;
                 // phase B of position t wrote y into stage sb; the stop is
                 // signalled through stop_pos (phase B never runs for it)
@@ -233,13 +243,15 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     if (*stop_pos <= t) { stop = true; break; }
                 if (stop) { PLR_STAMP(13); break; }
                 const long long jt = store_tile[sb];
-                if (STORE && !(jt == ntiles - 1 && last_ragged)) {
+                if (STORE && !(jt == ntiles - 1 && last_ragged))
                     bulk_store(prm.y + (size_t)jt * M, stB + (size_t)sb * SWL + kHalo, M * sizeof(T), pol);
-                    bulk_commit();
-                    bulk_wait_read<0>();                            // the store has read the stage
-                }
-                mbar_arrive(&emptyB[sb]);
+                bulk_commit();
+                bulk_wait_read<STQ - 1>();                          // stores up to t - STQ + 1 have read their stages
+                if (t - (STQ - 1) >= 0) mbar_arrive(&emptyB[(t - (STQ - 1)) % SB]);
             }
+            bulk_wait_read<0>();
+            for (int r = t - (STQ - 1); r < t; r++)
+                if (r >= 0) mbar_arrive(&emptyB[r % SB]);
             bulk_wait_all<0>();
             PLR_STAMP(14);
         }

@@ -34,11 +34,53 @@
 // as a full virtual tile whose positions beyond n are zero (zero inputs
 // before the start leave the zero state unchanged), and the map's halo
 // lies after the tile instead of before it.
+//
+// C > 1 (non-decaying signatures, forward, every tile resident): thread-block
+// clusters of C CTAs (C consecutive tiles) exchange their tile aggregates
+// through distributed shared memory, so the decoupled look-back runs over
+// CLUSTER records (one per C tiles): each CTA folds its in-cluster
+// predecessors' aggregates read over DSMEM (E_r), the cluster's rank 0
+// publishes the cluster aggregate and, after the look-back, its inclusive
+// carry, and tile r of cluster c enters with E_r + T(r m) G_{c-1}.  At 2^20
+// elements (273 tiles) the per-tile look-back read up to 272 records at once
+// from every CTA (a 3.3 us critical path, profiles/r03m_trace_small.jsonl);
+// the cluster look-back reads at most 36.  The carry algebra is P:527-542
+// applied to units of C tiles; padding CTAs beyond the last tile have zero
+// input (zero state), load and store nothing.
 #pragma once
 #include "plr_kernels.cuh"
 
 namespace plr {
 namespace dev {
+
+// ---- thread-block cluster / distributed shared memory ----------------------
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_arrive_release() { asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory"); }
+__device__ __forceinline__ void cluster_arrive_relaxed() { asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory"); }
+__device__ __forceinline__ void cluster_wait_acquire() { asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory"); }
+// value of type A at shared address p of CTA `rank` of this cluster
+template <typename A>
+__device__ __forceinline__ A ld_dsmem(const A* p, uint32_t rank) {
+    uint32_t a;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(smem_u32(p)), "r"(rank));
+    if constexpr (sizeof(A) == 8) {
+        unsigned long long v;
+        asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+        A out;
+        memcpy(&out, &v, 8);
+        return out;
+    } else {
+        uint32_t v;
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+        A out;
+        memcpy(&out, &v, 4);
+        return out;
+    }
+}
 
 // PLR_TRACE builds: globaltimer stamps of the launch's LAST tile (the end of
 // its critical path) into stats words 9..15 (plan made with PLR_STATS=1)
@@ -56,15 +98,19 @@ struct LayoutS {
     static constexpr size_t off_wagg = ((size_t)(kHalo + M) * sizeof(T) + 15) & ~(size_t)15;   // [W][kMaxK] A
     static constexpr size_t off_Pw = off_wagg + (size_t)W * kMaxK * sizeof(A);       // [W][kMaxK] A
     static constexpr size_t off_G = off_Pw + (size_t)W * kMaxK * sizeof(A);          // [kMaxK] A
-    static constexpr size_t off_bar = (off_G + kMaxK * sizeof(A) + 15) & ~(size_t)15;
+    static constexpr size_t off_Ac = off_G + kMaxK * sizeof(A);                     // [kMaxK] A: tile aggregate (DSMEM)
+    static constexpr size_t off_bar = (off_Ac + kMaxK * sizeof(A) + 15) & ~(size_t)15;
     static constexpr size_t off_tile = off_bar + 8;
     static constexpr size_t bytes = off_tile + 8;
 };
 
-template <typename T, typename A, int K, int P, int X, int W, bool REV = false>
+template <typename T, typename A, int K, int P, int X, int W, bool REV = false, int C = 1>
 __global__ void __launch_bounds__(W * 32, W >= 16 ? 1 : 2)
 plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = LayoutS<T, A, K, X, W>;
+    constexpr int LOGC = C >= 8 ? 3 : C >= 4 ? 2 : C >= 2 ? 1 : 0;
+    static_assert((1 << LOGC) == C && C <= 8, "cluster of 1, 2, 4 or 8 tiles");
+    static_assert(C == 1 || !REV, "cluster launches are forward only");
     constexpr int M = L::M;
     constexpr int LOGW = (W >= 16) ? 4 : (W >= 8) ? 3 : (W >= 4) ? 2 : (W >= 2) ? 1 : 0;
     static_assert((1 << LOGW) == W, "W must be a power of two");
@@ -258,6 +304,14 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (lane < W) sPw[lane * kMaxK + q] = lane == 0 ? A(0) : pw;
             At[q] = shfl_idx(u_[q], W - 1);
         }
+        if constexpr (C > 1) {
+            if (lane == 0) {
+                A* sAc = reinterpret_cast<A*>(smem + L::off_Ac);
+#pragma unroll
+                for (int q = 0; q < K; q++) sAc[q] = At[q];
+            }
+        }
+      if constexpr (C == 1) {
         A Gp[K];                                     // carries entering the tile
         if (j == 0) {
 #pragma unroll
@@ -297,6 +351,85 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         if (lane == 0) {
 #pragma unroll
             for (int q = 0; q < K; q++) sG[q] = Gp[q];
+        }
+      }
+    }
+    if constexpr (C > 1) {
+        // every CTA's aggregate is in its shared memory (barrier #1); warp 0
+        // reads the cluster's C aggregates, then arrives on barrier #2 (its
+        // shared memory may go once every CTA is past its DSMEM reads: the
+        // wait is at the end of the kernel)
+        __syncwarp();
+        cluster_arrive_release();
+        cluster_wait_acquire();
+        if (warp == 0) {
+            const uint32_t r = cluster_rank();               // == j mod C (tile = blockIdx.x)
+            A am[K];
+            const A* sAc = reinterpret_cast<const A*>(smem + L::off_Ac);
+#pragma unroll
+            for (int q = 0; q < K; q++) am[q] = lane < C ? ld_dsmem<A>(sAc + q, (uint32_t)lane) : A(0);
+            __syncwarp();
+            cluster_arrive_relaxed();
+            // E_r = sum_{i<r} T((r-1-i) m) A_i (zero carry into the cluster),
+            // Ac = the cluster aggregate; every lane folds redundantly
+            A E[K], Er[K];
+#pragma unroll
+            for (int q = 0; q < K; q++) { E[q] = A(0); Er[q] = A(0); }
+#pragma unroll
+            for (int i = 0; i < C; i++) {
+                A ai[K];
+#pragma unroll
+                for (int q = 0; q < K; q++) ai[q] = shfl_idx(am[q], i);
+                if ((uint32_t)i == r) {
+#pragma unroll
+                    for (int q = 0; q < K; q++) Er[q] = E[q];
+                }
+                matvec_acc<A, K>(ai, tb.Tm, E);              // E <- A_i + T(m) E
+#pragma unroll
+                for (int q = 0; q < K; q++) E[q] = ai[q];
+            }
+            const long long c = j / C;
+            A Gc[K];                                          // carries entering cluster c
+            if (c == 0) {
+#pragma unroll
+                for (int q = 0; q < K; q++) Gc[q] = prm.y_hist != nullptr ? A(prm.y_hist[K - 1 - q]) : A(0);
+            } else {
+                if (r == 0) publish_status<A, K, DECF>(prm.status, prm.status_mask, c, E, tagA, lane);
+                __shared__ unsigned long long s_lbst[kLbStatWords];   // debug counters (PLR_STATS=1)
+                const LbStats lbs{s_lbst};
+                lbs.init(lane);
+                __syncwarp();
+                lookback_generic<T, A, K, DECF, LOGC>(prm, tb, c, lane, tagA, tagI, Gc, lbs, 0, 0, 64, true);
+                __syncwarp();
+                lbs.flush(prm.stats, lane);
+            }
+            if (lane == 0) PLR_STAMP_LAST(13);
+            if (r == 0) {                                     // G_c = Ac + T(C m) G_{c-1}
+                A G[K];
+#pragma unroll
+                for (int q = 0; q < K; q++) G[q] = E[q];
+                matvec_acc<A, K>(G, tb.Tpow[LOGC], Gc);
+                publish_status<A, K, DECF>(prm.status, prm.status_mask, c, G, tagI, lane);
+            }
+            // carry entering tile j: E_r + T(r m) G_{c-1}, T(r m) from the binary powers T(2^b m)
+#pragma unroll
+            for (int b = 0; b < LOGC; b++) {
+                if ((r >> b) & 1u) {
+                    A t2[K];
+#pragma unroll
+                    for (int q = 0; q < K; q++) t2[q] = A(0);
+                    matvec_acc<A, K>(t2, tb.Tpow[b], Gc);
+#pragma unroll
+                    for (int q = 0; q < K; q++) Gc[q] = t2[q];
+                }
+            }
+            if (lane == 0) {
+#pragma unroll
+                for (int q = 0; q < K; q++) sG[q] = Er[q] + Gc[q];
+            }
+        } else {
+            __syncwarp();
+            cluster_arrive_relaxed();
         }
     }
     __syncthreads();
@@ -385,8 +518,9 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     }
     if (resident && tid == 0) {                      // the CTA's one ticket: the last one advances the state
         const long long rel = (long long)(atomicAdd(prm.ticket, 1ull) - s_tbase);
-        launch_state_advance(prm.ticket, rel, (unsigned long long)ntiles, s_tbase, epoch);
+        launch_state_advance(prm.ticket, rel, (unsigned long long)gridDim.x, s_tbase, epoch);
     }
+    if constexpr (C > 1) cluster_wait_acquire();     // barrier #2: no CTA of the cluster reads this smem any more
 }
 
 }  // namespace dev

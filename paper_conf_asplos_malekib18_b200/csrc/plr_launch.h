@@ -27,6 +27,7 @@ struct LaunchArgs {
     bool store;
     bool unit1 = false;                 // look-back units of one tile (small n): the *_u1 kernels
     bool reverse = false;               // the anticausal recurrence (REV kernels: small-n, DECAY)
+    bool cluster = false;               // small-n kernel: clusters of kSmallC tiles (cluster look-back)
     cudaStream_t stream;
     int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel
 };
@@ -62,6 +63,7 @@ cudaError_t launch_scan(const PlanTables& pt, const LaunchArgs& la);
 // geo_s, grid = ntiles (la.grid ignored); la.y == nullptr: reduce-only
 cudaError_t launch_small(const PlanTables& pt, const LaunchArgs& la);
 cudaError_t small_occupancy(const PlanTables& pt, int* ctas_per_sm);
+cudaError_t small_cluster_occupancy(const PlanTables& pt, int* clusters);   // co-resident clusters of kSmallC
 // the reduce-only kernel (plr_kernels_reduce.cuh): la.status = per-CTA record
 // scratch (kStatusMaxBytes each), la.grid CTAs over contiguous tile ranges of
 // kRedX * kRedW * 32 elements, la.y_tail = the K end-state outputs

@@ -13,6 +13,24 @@ cudaError_t launch_kp(const Tables<T, A>& tab, const LaunchArgs& la) {
     void (*kern)(const ScanParams<T, A>) = la.reverse ? &dev::plr_small_kernel<T, A, K, P, kSmallX, kSmallW, true>
                                                       : &dev::plr_small_kernel<T, A, K, P, kSmallX, kSmallW, false>;
     static_assert(L::bytes <= 48 * 1024, "small-n kernel needs no dynamic shared memory opt-in");
+    if (la.cluster) {                       // clusters of kSmallC tiles (forward, resident)
+        void (*kc)(const ScanParams<T, A>) = &dev::plr_small_kernel<T, A, K, P, kSmallX, kSmallW, false, kSmallC>;
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)((la.ntiles + kSmallC - 1) / kSmallC * kSmallC), 1, 1);
+        cfg.blockDim = dim3(kSmallW * 32, 1, 1);
+        cfg.dynamicSmemBytes = L::bytes;
+        cfg.stream = la.stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = kSmallC;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        if (la.occupancy_out != nullptr) return cudaOccupancyMaxActiveClusters(la.occupancy_out, kc, &cfg);
+        const ScanParams<T, A> prm = make_params(tab, la);
+        return cudaLaunchKernelEx(&cfg, kc, prm);
+    }
     if (la.occupancy_out != nullptr)
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(la.occupancy_out, kern, kSmallW * 32, L::bytes);
     const ScanParams<T, A> prm = make_params(tab, la);

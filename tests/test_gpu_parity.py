@@ -425,3 +425,45 @@ def test_reduce_kernel_end_state(cuda_plr, name, n):
     assert np.array_equal(xt, x[n - 4:])
     check(got.astype(np.float64) if sig.dtype == "float32" else got, ref[n - sig.k:], sig.dtype, "%s n=%d" % (name, n))
     plan.close()
+
+
+# ------------------------------------------------- small n: cluster launches --
+CLUSTER_SIGS = {s.name: s for s in workloads.TABLE1 if s.name in ("prefix", "tuple2", "tuple3", "order2", "order3")}
+CLUSTER_SIGS.update({s.name: s for s in (
+    workloads.Signature("order4", (1,), (4, -6, 4, -1), "int32", "4th-order prefix sum", "P:140-143"),
+    workloads.Signature("fir_order2", (3, -1, 2, 5), (2, -1), "int32", "FIR map + 2nd-order sum", "Eq. (1)"),
+    workloads.Signature("fsum", (1.0,), (1.0,), "float32", "float prefix sum (FLOAT class)", "P:97"))})
+
+
+@pytest.mark.parametrize("name", sorted(CLUSTER_SIGS))
+@pytest.mark.parametrize("cluster", ["1", "0"])
+def test_small_n_cluster_lookback(cuda_plr, name, cluster, monkeypatch):
+    """Non-decaying small-n launches run in clusters of 8 tiles whose
+    aggregates meet over DSMEM; the look-back runs over cluster records
+    (plr_kernels_small.cuh).  Tile counts around cluster boundaries (1, 2,
+    7, 8, 9, 16, 17, 64, 65, 273 and the most resident tiles) with ragged
+    tails, cluster launches on and off, against the oracle; continuation
+    with history enters the first cluster's carry."""
+    import torch
+    sig = CLUSTER_SIGS[name]
+    monkeypatch.setenv("PLR_SMALL_CLUSTER", cluster)
+    monkeypatch.setenv("PLR_SMALL_MAX", str(1 << 21))
+    ms = 3840
+    tiles = [1, 2, 7, 8, 9, 16, 17, 64, 65, 273, 295, 296]
+    sizes = sorted({t * ms - d for t in tiles for d in (0, 1)} | {2 * ms + 17, 9 * ms + 1})
+    x_all = workloads.host_input(max(sizes) + 64, sig.dtype, workloads.seed_for(13))
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=max(sizes) + 64)
+    for n in sizes:
+        x = x_all[:n].copy()
+        y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+        check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s n=%d cluster=%s" % (name, n, cluster))
+    # continuation: the second chunk starts from the first chunk's history
+    n1, n2 = 17 * ms + 5, 64 * ms + 3
+    x = x_all[:n1 + n2].copy()
+    ref = oracle.recurrence(x, sig.a, sig.b, sig.dtype)
+    y1 = plan(torch.from_numpy(x[:n1].copy()).cuda()).cpu().numpy()
+    xh = torch.from_numpy(x[max(0, n1 - plan.p):n1].copy()).cuda() if plan.p > 0 else None
+    yh = torch.from_numpy(y1[n1 - plan.k:].copy()).cuda()
+    y2 = plan.continue_(torch.from_numpy(x[n1:].copy()).cuda(), x_hist=xh, y_hist=yh).cpu().numpy()
+    check(np.concatenate([y1, y2]), ref, sig.dtype, "%s continuation cluster=%s" % (name, cluster))
+    plan.close()
