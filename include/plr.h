@@ -50,7 +50,7 @@
 extern "C" {
 #endif
 
-#define PLR_ABI_VERSION 3
+#define PLR_ABI_VERSION 4
 #define PLR_MAX_K 4            /* maximum order k supported by the kernels      */
 #define PLR_MAX_P 3            /* maximum feed-forward order p                  */
 #define PLR_PAYLOAD_BYTES 64   /* one rank's end-state record, see plr_reduce   */
@@ -111,6 +111,11 @@ typedef struct {
                                   rounds the input) relative to a Nyquist-frequency output
                                   (reading R20); 0 int                        */
     double nyquist_gain;       /* float: |H(-1)|, the gain at the Nyquist frequency; 0 int */
+    int small_clusters;        /* co-resident thread-block clusters of small-n CTAs (the
+                                  cluster look-back of non-decaying small launches); 0: none */
+    int small_cluster_ctas;    /* CTAs (tiles) per such cluster                        */
+    int small_ctas_per_sm;     /* CTAs per SM of the small-n kernel                    */
+    size_t small_max;          /* n <= small_max runs the small-n kernel               */
 } plr_plan_info;
 
 /* Create a plan.  a[0..p] = (a0, a-1, ..., a-p) (p = feed-forward order, so

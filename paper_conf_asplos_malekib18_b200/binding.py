@@ -64,7 +64,8 @@ class PlanInfo(ctypes.Structure):
                 ("fixup_len", ctypes.c_int64), ("n_max", _S), ("scratch_bytes", _S), ("ctas_per_sm", _I),
                 ("num_sms", _I), ("const_sig", _I),
                 ("tiles_per_unit", _I), ("kernel_kind", _I), ("acc_bits", _I), ("cond_bound", ctypes.c_double),
-                ("map_floor", ctypes.c_double), ("nyquist_gain", ctypes.c_double)]
+                ("map_floor", ctypes.c_double), ("nyquist_gain", ctypes.c_double),
+                ("small_clusters", _I), ("small_cluster_ctas", _I), ("small_ctas_per_sm", _I), ("small_max", _S)]
 
 
 class PLRError(RuntimeError):

@@ -93,13 +93,18 @@ static uint64_t unit1_waves() {
 // no pipeline).  Measured crossover against the
 // persistent kernels (profiles/r03e_sweep_auto.md vs r03c_sweep_big.md):
 // 2^21 for DECAY and first-order plans (single-hop / scalar look-back), 2^17
-// for k >= 2 non-decaying plans (their look-back over every predecessor
-// costs more than the persistent kernels' units beyond that).  PLR_SMALL_MAX
-// overrides it at plan creation (0: never).
-static size_t small_max_default(const PlanTables& pt) {
+// for k >= 2 non-decaying plans with the per-tile look-back (its reads of
+// every predecessor cost more than the persistent kernels' units beyond
+// that); with cluster launches (§6) the k >= 2 crossover is 2^20 or the
+// largest all-resident cluster launch if smaller (r03s: order3 at 2^20 15.3
+// us against 18.3 us on the re-read kernel, tuple2 14.8 / 15.1).
+// PLR_SMALL_MAX overrides it at plan creation (0: never).
+static size_t small_max_default(const PlanTables& pt, int small_clusters) {
     const char* e = std::getenv("PLR_SMALL_MAX");
     if (e != nullptr) return (size_t)std::strtoull(e, nullptr, 10);
-    return (pt.decay_flag || pt.k == 1) ? ((size_t)1 << 21) : ((size_t)1 << 17);
+    if (pt.decay_flag || pt.k == 1) return (size_t)1 << 21;
+    const size_t cl = (size_t)small_clusters * kSmallC * (size_t)pt.geo_s.tile();
+    return small_clusters > 0 ? std::max(std::min(cl, (size_t)1 << 20), (size_t)1 << 17) : ((size_t)1 << 17);
 }
 
 // ============================================================ helpers =====
@@ -462,14 +467,16 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
             if ((e = cudaMalloc(&plan->d_rd, rb)) != cudaSuccess) return bail(e, "alloc reduce records");
         }
     }
-    plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default(plan->pt)) : 0;
     plan->small_ctas = small_ctas;
     if (!plan->pt.decay_s && small_ctas >= 1) {
         if ((e = small_cluster_occupancy(plan->pt, &plan->small_clusters)) != cudaSuccess) {
             (void)cudaGetLastError();                          // no cluster launches on this device
             plan->small_clusters = 0;
+            if (std::getenv("PLR_DEBUG") != nullptr)
+                std::fprintf(stderr, "plr: cluster occupancy query failed: %s\n", cudaGetErrorString(e));
         }
     }
+    plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default(plan->pt, plan->small_clusters)) : 0;
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
     // Two status arrays: the persistent kernels' (their tiles up to n_max)
@@ -607,6 +614,10 @@ plr_status plr_plan_get_info(const plr_plan* plan, plr_plan_info* info) {
     info->cond_bound = plan->pt.dtype == PLR_FLOAT32 ? plan->pt.cond_bound : 0.0;
     info->map_floor = plan->pt.dtype == PLR_FLOAT32 ? plan->pt.map_floor : 0.0;
     info->nyquist_gain = plan->pt.dtype == PLR_FLOAT32 ? plan->pt.nyquist_gain : 0.0;
+    info->small_clusters = plan->small_clusters;
+    info->small_cluster_ctas = kSmallC;
+    info->small_ctas_per_sm = plan->small_ctas;
+    info->small_max = plan->small_max;
     return PLR_OK;
 }
 

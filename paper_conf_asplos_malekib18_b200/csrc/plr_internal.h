@@ -127,7 +127,7 @@ constexpr int kSmallW = PLR_SMALL_W;
 // clusters of kSmallC tiles exchange aggregates over DSMEM, the look-back
 // runs over cluster records (plr_kernels_small.cuh)
 #ifndef PLR_SMALL_C
-#define PLR_SMALL_C 8
+#define PLR_SMALL_C 4
 #endif
 constexpr int kSmallC = PLR_SMALL_C;
 // reduce-only kernel geometry (plr_kernels_reduce.cuh): X = 31, W = 8

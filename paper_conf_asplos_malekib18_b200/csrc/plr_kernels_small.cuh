@@ -44,7 +44,8 @@
 // carry, and tile r of cluster c enters with E_r + T(r m) G_{c-1}.  At 2^20
 // elements (273 tiles) the per-tile look-back read up to 272 records at once
 // from every CTA (a 3.3 us critical path, profiles/r03m_trace_small.jsonl);
-// the cluster look-back reads at most 36.  The carry algebra is P:527-542
+// with clusters of 4 (71 co-resident on B200; clusters of 8 fit only 33,
+// GPC fragmentation) the look-back reads at most 70.  The carry algebra is P:527-542
 // applied to units of C tiles; padding CTAs beyond the last tile have zero
 // input (zero state), load and store nothing.
 #pragma once

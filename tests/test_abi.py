@@ -28,7 +28,7 @@ def test_exports_every_declared_symbol():
     for s in syms:
         assert hasattr(plr.lib, s), s
     assert set(syms) == set(plr.binding.EXPORTED)
-    assert plr.abi_version() == 3
+    assert plr.abi_version() == 4
 
 
 @pytest.mark.parametrize("a,b,dtype,code", [

@@ -449,7 +449,16 @@ def test_small_n_cluster_lookback(cuda_plr, name, cluster, monkeypatch):
     monkeypatch.setenv("PLR_SMALL_CLUSTER", cluster)
     monkeypatch.setenv("PLR_SMALL_MAX", str(1 << 21))
     ms = 3840
-    tiles = [1, 2, 7, 8, 9, 16, 17, 64, 65, 273, 295, 296]
+    probe = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=1 << 21)
+    info = probe.info
+    probe.close()
+    c = info["small_cluster_ctas"]
+    top = info["small_clusters"] * c                     # most tiles of a cluster launch
+    assert top >= 64, "cluster launches unavailable: %s" % info
+    # tile counts around cluster boundaries, up to the largest cluster launch
+    # and one tile beyond it (the per-tile look-back again)
+    tiles = sorted({t for t in (1, 2, c - 1, c, c + 1, 2 * c, 2 * c + 1, 64, 65, 273, top - 1, top, top + 1)
+                    if 1 <= t <= top + 1})
     sizes = sorted({t * ms - d for t in tiles for d in (0, 1)} | {2 * ms + 17, 9 * ms + 1})
     x_all = workloads.host_input(max(sizes) + 64, sig.dtype, workloads.seed_for(13))
     plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=max(sizes) + 64)

@@ -1,7 +1,7 @@
-# round-2 batch j: the measurement set at HEAD -- bench (+ reference arm), launch list, ncu captures
+# the measurement set at HEAD -- bench (+ reference arm), launch list, ncu captures
 # (bench kernels, fp64 DECAY, reduce-only), worst float error, ablation, size sweep, reduce timing
 set -x
-TAG=${TAG:-r03j}
+TAG=${TAG:-head}
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/${TAG}_smi.txt
 timeout 1200 python -m pytest tests -m gpu -q --timeout 900 -p no:cacheprovider > gpurun_out/${TAG}_pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/${TAG}_pytest_gpu.log
