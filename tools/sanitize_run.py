@@ -1,6 +1,8 @@
 """Small-grid launches of every scan-kernel family for compute-sanitizer
 (memcheck / racecheck / synccheck): a few tiles each, checked against the
-oracle.  Usage: compute-sanitizer --tool T python tools/sanitize_run.py"""
+oracle.  Usage: compute-sanitizer --tool T python tools/sanitize_run.py
+(PLR_SMALL_MAX=0: the persistent kernels; default: the small-n kernel,
+cluster launches for the non-decaying rows)"""
 import os
 import sys
 
@@ -25,7 +27,11 @@ for name, n in CASES:
         ok = np.array_equal(y, ref)
     else:
         ok = float(np.max(np.abs(y - ref) / np.maximum(1, np.abs(ref)))) <= 1e-4
-    print(name, n, plan.kernel_name(), "ok" if ok else "MISMATCH", flush=True)
+    info = plan.info
+    kern = plan.kernel_name() if n > info["small_max"] else (
+        "plr_small_kernel" + (" (clusters of %d)" % info["small_cluster_ctas"]
+                              if info["small_clusters"] > 0 and os.environ.get("PLR_SMALL_CLUSTER", "1") != "0" else ""))
+    print(name, n, kern, "ok" if ok else "MISMATCH", flush=True)
     bad += not ok
     plan.close()
 torch.cuda.synchronize()
