@@ -23,6 +23,7 @@
 // (a1-a4) of tile i+D before phase B (a6-a7) of tile i, so the look-back
 // latency of a tile overlaps D tiles of compute.
 #pragma once
+#include <cstdio>
 #include <cuda_runtime.h>
 #include <cstdint>
 
@@ -57,6 +58,39 @@ __device__ __forceinline__ void launch_state_advance(unsigned long long* tk, lon
 #else
 #define PLR_STAMP(i) do { } while (0)
 #endif
+
+// ------------------------------------------------------- deadlock trap ----
+// PLR_DEADLOCK_TRAP builds (tests / stress variants, never the product
+// library): every spin / poll loop of the kernels carries a SpinGuard that
+// reads %globaltimer and, after PLR_DEADLOCK_NS of waiting at one site,
+// prints the site, block and thread and executes trap -- a lost arrival or
+// an unpublished status record becomes a launch error with a location
+// instead of a hung GPU.  Sites: 1 mbar_wait, 2 mbar_wait_poll, 3
+// mbar_wait_or_stop, 4 re-read loader B, 5 re-read storer, 6 generic
+// look-back poll, 7 DECAY single-hop poll (plr_scan_kernel), 8 (dect
+// kernel), 9 (small-n kernel).  Product builds: an empty struct, no code.
+#ifndef PLR_DEADLOCK_NS
+#define PLR_DEADLOCK_NS 2000000000ull
+#endif
+
+struct SpinGuard {
+#ifdef PLR_DEADLOCK_TRAP
+    unsigned long long t0 = 0;
+    __device__ __forceinline__ void operator()(int site) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        if (t0 == 0) {
+            t0 = t;
+        } else if (t - t0 > (unsigned long long)PLR_DEADLOCK_NS) {
+            printf("plr deadlock trap: site %d block %d thread %d waited %llu ns\n", site, (int)blockIdx.x,
+                   (int)threadIdx.x, t - t0);
+            __trap();
+        }
+    }
+#else
+    __device__ __forceinline__ void operator()(int) {}
+#endif
+};
 
 // ---------------------------------------------------------------- PTX ------
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -135,7 +169,9 @@ __device__ __forceinline__ bool mbar_poll(uint64_t* bar, uint32_t parity) {
 // warp that the awaited arrival depends on (those lanes use mbar_poll).
 __device__ __forceinline__ bool mbar_wait_or_stop(uint64_t* bar, uint32_t parity, const volatile int* stop_pos,
                                                   int pos, const volatile int* draining) {
+    SpinGuard guard;
     for (;;) {
+        guard(3);
         if (mbar_test(bar, parity)) return true;
         if (*stop_pos <= pos) return false;
         if (*draining) {
@@ -146,14 +182,16 @@ __device__ __forceinline__ bool mbar_wait_or_stop(uint64_t* bar, uint32_t parity
     }
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    while (!mbar_try_wait_sleep(bar, parity, PLR_WAIT_HINT_NS)) { }
+    SpinGuard guard;
+    while (!mbar_try_wait_sleep(bar, parity, PLR_WAIT_HINT_NS)) guard(1);
 }
 // wait without a suspend hint, for lanes of a warp whose lanes play
 // different roles (loader / storer lanes of the producer warp): a lane
 // suspended for long in try_wait can hold back a diverged sibling lane that
 // the awaited arrival depends on (loader B waits on the storer's emptyB)
 __device__ __forceinline__ void mbar_wait_poll(uint64_t* bar, uint32_t parity) {
-    while (!mbar_try_wait(bar, parity)) { }
+    SpinGuard guard;
+    while (!mbar_try_wait(bar, parity)) guard(2);
 }
 // TMA 1D bulk copy global -> shared, completion on an mbarrier (UBLKCP).
 __device__ __forceinline__ void bulk_load(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar,
@@ -439,6 +477,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
 #endif
     int ns = PLR_LB_NS0;
     unsigned long long n_win = 0, n_wait = 0;
+    SpinGuard guard;
     long long c_load = 0, c_fold = 0;
     for (;;) {
         n_win++;
@@ -530,6 +569,7 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
             if (dN >= (1 << 30)) ltpl = kLogT;         // nothing pending: widen to the full window
         } else {
             n_wait++;                                  // nearest tile not ready yet
+            guard(6);
             const long long cw = clock64();
             __nanosleep(ns);
             c_wait += clock64() - cw;
@@ -735,7 +775,9 @@ plr_scan_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 A v[K];
                 if (lane == 0) {
                     int ns = 64;
+                    SpinGuard guard;
                     while (read_status<A, K, DEC>(prm.status, prm.status_mask, j - 1, v, tagA, tagI) != 2) {
+                        guard(7);
                         __nanosleep(ns);
                         ns = ns < 256 ? 2 * ns : ns;
                     }

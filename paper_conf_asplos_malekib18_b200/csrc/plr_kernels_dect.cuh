@@ -175,7 +175,9 @@ plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 A v[K];
                 if (lane == 0) {
                     int ns = 64;
+                    SpinGuard guard;
                     while (read_status<A, K, DEC>(prm.status, prm.status_mask, j - 1, v, tagA, tagI) != 2) {
+                        guard(8);
                         __nanosleep(ns);
                         ns = ns < 256 ? 2 * ns : ns;
                     }

@@ -210,8 +210,11 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 const int slot = f % NS;
                 const uint32_t par = (uint32_t)((f / NS) & 1);
                 bool stop = false;
-                while (!mbar_poll(&agg_bar[slot], par))
+                SpinGuard guard;
+                while (!mbar_poll(&agg_bar[slot], par)) {
+                    guard(4);
                     if (*stop_pos <= f) { stop = true; break; }
+                }
                 const long long j = stop ? ntiles : slot_tile[slot];
                 if (j >= ntiles) break;
                 if (f >= SB) mbar_wait_poll(&emptyB[sb], (uint32_t)(((f / SB) - 1) & 1));
@@ -239,8 +242,11 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 // signalled through stop_pos (phase B never runs for it)
                 const uint32_t par = (uint32_t)((t / SB) & 1);
                 bool stop = false;
-                while (!mbar_poll(&yfull[sb], par))
+                SpinGuard guard;
+                while (!mbar_poll(&yfull[sb], par)) {
+                    guard(5);
                     if (*stop_pos <= t) { stop = true; break; }
+                }
                 if (stop) { PLR_STAMP(13); break; }
                 const long long jt = store_tile[sb];
                 if (STORE && !(jt == ntiles - 1 && last_ragged))

@@ -322,7 +322,9 @@ plr_small_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             A g[K];
             if (lane == 0) {
                 int ns = 32;
+                SpinGuard guard;
                 while (read_status<A, K, DECF>(prm.status, prm.status_mask, j - 1, g, tagA, tagI) != 2) {
+                    guard(9);
                     __nanosleep(ns);
                     ns = ns < 128 ? 2 * ns : ns;
                 }

@@ -1,5 +1,6 @@
 """Time signatures at n (no debug stats): ms, GB/s, fraction of an in-run memcpy.
-Usage: python tools/time_sigs.py [n] [sig,sig,...]   (PLR_LIB selects a variant library)"""
+Usage: python tools/time_sigs.py [n] [sig,sig,...] [scan|reverse|bidir]   (PLR_LIB selects a variant library)
+reverse: the anticausal pass; bidir: forward + anticausal (two passes, 16 B per element counted)"""
 import os
 import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -8,7 +9,9 @@ import paper_conf_asplos_malekib18_b200 as plr  # noqa: E402
 import workloads  # noqa: E402
 
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 1 << 30
-names = sys.argv[2].split(",") if len(sys.argv) > 2 else [s.name for s in workloads.TABLE1]
+names = sys.argv[2].split(",") if len(sys.argv) > 2 and sys.argv[2] else [s.name for s in workloads.TABLE1]
+mode = sys.argv[3] if len(sys.argv) > 3 else "scan"
+passes = 2 if mode == "bidir" else 1
 xi = workloads.device_input(n, "int32", 1)
 xf = workloads.device_input(n, "float32", 2)
 y = torch.empty_like(xi)
@@ -34,7 +37,13 @@ for name in names:
     x = xi if sig.dtype == "int32" else xf
     yy = y if sig.dtype == "int32" else y.view(torch.float32)
     plan = plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
-    ms = timed(lambda: plan(x, yy))
-    print("%-7s %8.3f ms %7.1f GB/s  %.3f of memcpy  %s" % (name, ms, n * 8 / ms / 1e6, ms_cp / ms,
+    if mode == "reverse":
+        ms = timed(lambda: plan.reverse(x, yy))
+    elif mode == "bidir":
+        tmp = torch.empty_like(yy)
+        ms = timed(lambda: plan.bidirectional(x, yy, tmp=tmp))
+    else:
+        ms = timed(lambda: plan(x, yy))
+    print("%-7s %8.3f ms %7.1f GB/s  %.3f of memcpy  %s" % (name, ms, passes * n * 8 / ms / 1e6, passes * ms_cp / ms,
           {k: plan.info[k] for k in ("ctas_per_sm", "cls", "tile_elems")}), flush=True)
     plan.close()
