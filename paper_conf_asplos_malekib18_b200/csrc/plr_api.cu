@@ -260,11 +260,9 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         plan->epoch = 0;
         plan->dirty = false;
     }
-    // small n: one CTA per tile, no pipeline; the anticausal pass of a
-    // non-DECAY or fp64-accumulation plan runs the small-n kernel at every
-    // size (the in-place DECAY kernel's fp64 footprint at the wide geometry
-    // exceeds shared memory)
-    if (n <= plan->small_max || (reverse && (!plan->pt.decay_flag || plan->pt.acc64))) {
+    // small n: one CTA per tile, no pipeline (the anticausal pass too; beyond
+    // small_max it runs the REV instantiation of the plan's persistent kernel)
+    if (n <= plan->small_max) {
         const uint64_t ms = (uint64_t)plan->pt.geo_s.tile();
         plan->epoch++;
         LaunchArgs la;
@@ -326,7 +324,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.lane_T = plan->d_lane;
     la.stats = plan->d_stats;
     la.grid = (int)grid;
-    la.sig = plan->sig_kernel ? plan->pt.sig_id : 0;
+    la.sig = (plan->sig_kernel && !reverse) ? plan->pt.sig_id : 0;   // REV kernels read the parameter tables
     la.store = store;
     la.unit1 = unit1;
     la.reverse = reverse;
@@ -480,12 +478,10 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
     // Two status arrays: the persistent kernels' (their tiles up to n_max)
-    // and the small-n kernel's (its tiles up to small_max -- up to n_max for
-    // plans whose anticausal pass runs the small-n kernel at every size).
+    // and the small-n kernel's (its tiles up to small_max).
     // One shared array sized for the small tiles doubled the persistent
     // kernels' and cost their forward pass ~3 % at 2^30 (r03e/r03f A/B).
-    const bool rev_small = !plan->pt.decay_flag || plan->pt.acc64;
-    const uint64_t small_tiles = std::max<uint64_t>(1, ((rev_small ? n_max : plan->small_max) + ms - 1) / ms);
+    const uint64_t small_tiles = std::max<uint64_t>(1, (plan->small_max + ms - 1) / ms);
     if (plan->max_tiles > (1ull << 31) || small_tiles > (1ull << 31)) {
         plr_plan_destroy(plan);
         return fail(PLR_ERR_SIZE, "n_max too large");

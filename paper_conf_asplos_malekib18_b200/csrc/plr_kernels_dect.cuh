@@ -50,7 +50,11 @@ struct LayoutDT {
     static constexpr size_t bytes = off_lbstat + kMaxNL * kLbStatWords * 8;
 };
 
-template <typename T, typename A, int K, int P, int X, int W, int SL, int ST, int D, int MINB>
+// REV: the anticausal recurrence (plr_kernels_small.cuh): ticket j is
+// original tile ntiles-1-j read back to front, the ragged tile first (a
+// virtual full tile, zero beyond n), the map's halo after the tile (load
+// stage layout [tile][halo]); y goes into the store ring in original order.
+template <typename T, typename A, int K, int P, int X, int W, int SL, int ST, int D, int MINB, bool REV = false>
 __global__ void __launch_bounds__((W + 2) * 32, MINB)
 plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     constexpr int NT = D + 1;                                   // parked tiles (phase-B lag D)
@@ -95,6 +99,10 @@ plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
     const Tables<T, A>& tb = prm.tab;
+    // the tile the compute warps load element by element (REV: the first)
+    auto is_ragged = [&](long long j) -> bool { return last_ragged && j == (REV ? 0 : ntiles - 1); };
+    // first element of tile j in the arrays (REV: original tile ntiles-1-j)
+    auto tile_start = [&](long long j) -> long long { return (REV ? ntiles - 1 - j : j) * (long long)M; };
 
     const unsigned long long tbase = ld_volatile_u64(prm.ticket + 1);
     const uint32_t epoch = (uint32_t)ld_volatile_u64(prm.ticket + 2) + 1u;
@@ -125,9 +133,18 @@ plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     mbar_arrive(&full_L[s]);
                     break;
                 }
-                if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_L[s]); continue; }   // compute loads it
+                if (is_ragged(j)) { mbar_arrive(&full_L[s]); continue; }   // compute loads it
                 T* st = lstage + (size_t)s * SWL;
-                if (j == 0) {
+                if (REV) {                                      // the tile, its halo after it (zero beyond n)
+                    const long long o = tile_start(j);
+#pragma unroll
+                    for (int q = 0; q < kHalo; q++) {
+                        const unsigned long long i = (unsigned long long)(o + M + q);
+                        st[M + q] = (q < P && i < n) ? prm.x[i] : T(0);
+                    }
+                    mbar_arrive_tx(&full_L[s], M * sizeof(T));
+                    bulk_load(st, prm.x + (size_t)o, M * sizeof(T), &full_L[s], pol);
+                } else if (j == 0) {
 #pragma unroll
                     for (int q = 0; q < kHalo; q++)
                         st[q] = (q >= kHalo - P && prm.x_hist != nullptr) ? prm.x_hist[q - (kHalo - P)] : T(0);
@@ -144,8 +161,8 @@ plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 mbar_wait_poll(&full_T[sT], (uint32_t)((t / ST) & 1));
                 const long long jt = store_tile[sT];
                 if (jt >= ntiles) break;
-                if (!(jt == ntiles - 1 && last_ragged)) {
-                    bulk_store(prm.y + (size_t)jt * M, tstage + (size_t)sT * M, M * sizeof(T), pol);
+                if (!is_ragged(jt)) {
+                    bulk_store(prm.y + (size_t)tile_start(jt), tstage + (size_t)sT * M, M * sizeof(T), pol);
                     bulk_commit();
                     bulk_wait_read<0>();                            // the store has read the stage
                 }
@@ -210,11 +227,25 @@ plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (tid == 0) { slot_tile[slot] = j; mbar_arrive(&agg_bar[slot]); }
             return j;
         }
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         const long long g0 = j * (long long)M + (long long)tid * X;
         // a1: my X inputs (+ P halo), then the load stage goes back to the loader
         T xv[X + P];
-        if (!ragged) {
+        if (REV) {                                              // positions v: element o + M-1-v
+            const int v0 = tid * X - P;
+            if (!ragged) {
+                const T* st = lstage + (size_t)s * SWL;
+#pragma unroll
+                for (int q = 0; q < X + P; q++) xv[q] = st[M - 1 - (v0 + q)];
+            } else {
+                const long long o = tile_start(j);
+#pragma unroll
+                for (int q = 0; q < X + P; q++) {
+                    const unsigned long long i = (unsigned long long)(o + M - 1 - (v0 + q));
+                    xv[q] = i < n ? prm.x[i] : T(0);
+                }
+            }
+        } else if (!ragged) {
             const T* base = lstage + (size_t)s * SWL + kHalo + tid * X;
 #pragma unroll
             for (int q = 0; q < P; q++) xv[q] = base[q - P];
@@ -319,7 +350,7 @@ plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         const int sT = it % ST;
         mbar_wait(&carry_bar[slot], (uint32_t)((it / NT) & 1));
         const long long j = slot_tile[slot];
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         const long long g0 = j * (long long)M + (long long)tid * X;
         uint32_t w[CW];
         tmem_ld_n<CW>(tmem_w + (uint32_t)(slot * WQ * CW), w);
@@ -361,17 +392,17 @@ plr_scan_dect_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         // a7: into the store ring (ragged tile: direct stores)
         mbar_wait(&empty_T[sT], (uint32_t)(((it / ST) & 1) ^ 1));
         if (!ragged) {
-            T* base = tstage + (size_t)sT * M + tid * X;
+            T* stt = tstage + (size_t)sT * M;
 #pragma unroll
-            for (int u = 0; u < X; u++) base[u] = yv[u];
+            for (int u = 0; u < X; u++) stt[REV ? M - 1 - (tid * X + u) : tid * X + u] = yv[u];
         } else {
 #pragma unroll
             for (int u = 0; u < X; u++) {
-                const long long i = g0 + u;
+                const long long i = REV ? tile_start(j) + M - 1 - (tid * X + u) : g0 + u;
                 if ((unsigned long long)i < n) prm.y[i] = yv[u];
             }
         }
-        if (prm.y_tail != nullptr) {
+        if (!REV && prm.y_tail != nullptr) {
             const long long lo = (long long)n - K;
             if (g0 + X > lo && g0 < (long long)n) {
 #pragma unroll

@@ -68,8 +68,12 @@ struct LayoutR {
 template <typename A, int K>
 struct RrCols { static constexpr int CW = K * AWords<A>::N; };
 
+// REV: the anticausal recurrence (plr_kernels_small.cuh): ticket j is
+// original tile ntiles-1-j read back to front, the ragged tile first (a
+// virtual full tile, zero beyond n), the map's halo after the tile (stage
+// layout [tile][halo]); phase B writes y into the stage in original order.
 template <typename T, typename A, int K, int P, int X, int W, int SA, int SB, int NS, int NL, int G, bool STORE,
-          int SIG>
+          int SIG, bool REV = false>
 __global__ void __launch_bounds__((W + 1 + NL) * 32, 1)
 plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = LayoutR<T, A, K, X, W, SA, SB, NS>;
@@ -120,6 +124,11 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const long long ntiles = (long long)prm.ntiles;
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
+    static_assert(!REV || STORE, "the anticausal pass always stores");
+    // the tile the compute warps load element by element (REV: the first)
+    auto is_ragged = [&](long long j) -> bool { return last_ragged && j == (REV ? 0 : ntiles - 1); };
+    // first element of tile j in the arrays (REV: original tile ntiles-1-j)
+    auto tile_start = [&](long long j) -> long long { return (REV ? ntiles - 1 - j : j) * (long long)M; };
     // SIG != 0: the signature's tables are compile-time constants (plr_constsig.cuh)
     constexpr Tables<T, A> kTab = const_tables<T, A>(SIG, X, W, G);
     static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
@@ -155,7 +164,16 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     };
     // TMA load of tile j (with its P-word halo) into stage st, completion on bar
     auto load_tile = [&](T* st, long long j, uint64_t* bar, uint64_t pol) {
-        if (j == 0) {
+        if (REV) {                                              // the tile, its halo after it (zero beyond n)
+            const long long o = tile_start(j);
+#pragma unroll
+            for (int q = 0; q < kHalo; q++) {
+                const unsigned long long i = (unsigned long long)(o + M + q);
+                st[M + q] = (q < P && i < n) ? prm.x[i] : T(0);
+            }
+            mbar_arrive_tx(bar, M * sizeof(T));
+            bulk_load(st, prm.x + (size_t)o, M * sizeof(T), bar, pol);
+        } else if (j == 0) {
 #pragma unroll
             for (int q = 0; q < kHalo; q++)
                 st[q] = (q >= kHalo - P && prm.x_hist != nullptr) ? prm.x_hist[q - (kHalo - P)] : T(0);
@@ -195,7 +213,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     mbar_arrive(&fullA[s]);
                     break;
                 }
-                if (j == ntiles - 1 && last_ragged) { mbar_arrive(&fullA[s]); continue; }   // compute loads it
+                if (is_ragged(j)) { mbar_arrive(&fullA[s]); continue; }   // compute loads it
                 load_tile(stA + (size_t)s * SWL, j, &fullA[s], pol);
             }
         } else if (lane == 1) {                                     // loader B (L2)
@@ -218,7 +236,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 const long long j = stop ? ntiles : slot_tile[slot];
                 if (j >= ntiles) break;
                 if (f >= SB) mbar_wait_poll(&emptyB[sb], (uint32_t)(((f / SB) - 1) & 1));
-                if (j == ntiles - 1 && last_ragged) { mbar_arrive(&fullB[sb]); continue; }
+                if (is_ragged(j)) { mbar_arrive(&fullB[sb]); continue; }
                 if (!covers_tail(j)) { mbar_arrive(&fullB[sb]); continue; }   // reduce-only: phase B skipped
                 load_tile(stB + (size_t)sb * SWL, j, &fullB[sb], pol);
             }
@@ -249,8 +267,9 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 }
                 if (stop) { PLR_STAMP(13); break; }
                 const long long jt = store_tile[sb];
-                if (STORE && !(jt == ntiles - 1 && last_ragged))
-                    bulk_store(prm.y + (size_t)jt * M, stB + (size_t)sb * SWL + kHalo, M * sizeof(T), pol);
+                if (STORE && !is_ragged(jt))
+                    bulk_store(prm.y + (size_t)tile_start(jt), stB + (size_t)sb * SWL + (REV ? 0 : kHalo),
+                               M * sizeof(T), pol);
                 bulk_commit();
                 bulk_wait_read<STQ - 1>();                          // stores up to t - STQ + 1 have read their stages
                 if (t - (STQ - 1) >= 0) mbar_arrive(&emptyB[(t - (STQ - 1)) % SB]);
@@ -368,7 +387,20 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // for the ragged last tile
     auto read_x = [&](const T* st, long long j, bool ragged, T (&xv)[X + P]) {
         const long long g0 = j * (long long)M + (long long)tid * X;
-        if (!ragged) {
+        if (REV) {                                              // positions v: element o + M-1-v
+            const int v0 = tid * X - P;
+            if (!ragged) {
+#pragma unroll
+                for (int q = 0; q < X + P; q++) xv[q] = st[M - 1 - (v0 + q)];
+            } else {
+                const long long o = tile_start(j);
+#pragma unroll
+                for (int q = 0; q < X + P; q++) {
+                    const unsigned long long i = (unsigned long long)(o + M - 1 - (v0 + q));
+                    xv[q] = i < n ? prm.x[i] : T(0);
+                }
+            }
+        } else if (!ragged) {
             const T* base = st + kHalo + tid * X;
 #pragma unroll
             for (int q = 0; q < P; q++) xv[q] = base[q - P];
@@ -402,27 +434,67 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (tid == 0) { slot_tile[slot] = j; *stop_pos = it; mbar_arrive(&agg_bar[slot]); }
             return j;
         }
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         T xv[X + P];
         read_x(stA + (size_t)s * SWL, j, ragged, xv);
         mbar_arrive(&emptyA[s]);                                // the stage may be refilled
         // a2: chunk end state with zero state (only the last K values matter)
-        A hist[K];
-#pragma unroll
-        for (int r = 0; r < K; r++) hist[r] = A(0);
-#pragma unroll
-        for (int u = 0; u < X; u++) {
-            A acc = cvt<A, T>(fir(xv, u));
-#pragma unroll
-            for (int r = K; r >= 1; r--)
-                if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
-#pragma unroll
-            for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
-            hist[0] = acc;
-        }
+#ifndef PLR_RR_SPLIT
+#define PLR_RR_SPLIT 0
+#endif
         A v[K];
+        if constexpr (PLR_RR_SPLIT && sizeof(A) == sizeof(T) && X >= 2 * K + 1) {
+            // two independent zero-state chains over [0, H) and [H, X) (twice
+            // the instruction-level parallelism of the serial chain), joined
+            // by the end state = h2 + T(X - H) h1, T(L)[q][r] = h^(r+1)_{L-1-q}
+            // = H[L-1-q][r] (Sec. 2.1)
+            constexpr int H = X / 2, H2 = X - H;
+            A h1[K], h2[K];
 #pragma unroll
-        for (int q = 0; q < K; q++) v[q] = hist[q];
+            for (int r = 0; r < K; r++) { h1[r] = A(0); h2[r] = A(0); }
+#pragma unroll
+            for (int u = 0; u < H2; u++) {
+                if (u < H) {
+                    A acc = cvt<A, T>(fir(xv, u));
+#pragma unroll
+                    for (int r = K; r >= 1; r--)
+                        if (u - r >= 0) acc = mad(tb.c[r - 1], h1[r - 1], acc);
+#pragma unroll
+                    for (int r = K - 1; r >= 1; r--) h1[r] = h1[r - 1];
+                    h1[0] = acc;
+                }
+                A acc2 = cvt<A, T>(fir(xv, H + u));
+#pragma unroll
+                for (int r = K; r >= 1; r--)
+                    if (u - r >= 0) acc2 = mad(tb.c[r - 1], h2[r - 1], acc2);
+#pragma unroll
+                for (int r = K - 1; r >= 1; r--) h2[r] = h2[r - 1];
+                h2[0] = acc2;
+            }
+#pragma unroll
+            for (int q = 0; q < K; q++) {
+                A acc = h2[q];
+#pragma unroll
+                for (int r = 0; r < K; r++) acc = mad(cvt<A, T>(tb.H[H2 - 1 - q][r]), h1[r], acc);
+                v[q] = acc;
+            }
+        } else {
+            A hist[K];
+#pragma unroll
+            for (int r = 0; r < K; r++) hist[r] = A(0);
+#pragma unroll
+            for (int u = 0; u < X; u++) {
+                A acc = cvt<A, T>(fir(xv, u));
+#pragma unroll
+                for (int r = K; r >= 1; r--)
+                    if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
+#pragma unroll
+                for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
+                hist[0] = acc;
+            }
+#pragma unroll
+            for (int q = 0; q < K; q++) v[q] = hist[q];
+        }
         // a3: warp inclusive scan with T(X * 2^s)
 #pragma unroll
         for (int s2 = 0; s2 < 5; s2++) {
@@ -503,7 +575,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             mbar_arrive(&yfull[sb]);
             return;
         }
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         const long long g0 = j * (long long)M + (long long)tid * X;
         uint32_t w[CW];
         tmem_ld_n<CW>(tmem_w + (uint32_t)(slot * WQ * CW), w);
@@ -543,18 +615,17 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         // a7: y into the stage (TMA store by the storer) or global (ragged)
         if (!ragged) {
             if (STORE) {
-                T* base = st + kHalo + tid * X;
 #pragma unroll
-                for (int u = 0; u < X; u++) base[u] = yv[u];
+                for (int u = 0; u < X; u++) st[REV ? M - 1 - (tid * X + u) : kHalo + tid * X + u] = yv[u];
             }
         } else if (STORE) {
 #pragma unroll
             for (int u = 0; u < X; u++) {
-                const long long i = g0 + u;
+                const long long i = REV ? tile_start(j) + M - 1 - (tid * X + u) : g0 + u;
                 if ((unsigned long long)i < n) prm.y[i] = yv[u];
             }
         }
-        if (prm.y_tail != nullptr) {
+        if (!REV && prm.y_tail != nullptr) {
             const long long lo = (long long)n - K;
             if (g0 + X > lo && g0 < (long long)n) {
 #pragma unroll

@@ -153,8 +153,12 @@ struct LayoutT {
 template <typename A, int K, int X>
 struct TmemCols { static constexpr int CW = X + K * AWords<A>::N; };
 
+// REV: the anticausal recurrence (plr_kernels_small.cuh): ticket j is
+// original tile ntiles-1-j read back to front, the ragged tile first (a
+// virtual full tile, zero beyond n), the map's halo after the tile (load
+// stage layout [tile][halo]); y goes into the store ring in original order.
 template <typename T, typename A, int K, int P, int X, int W, int SL, int ST, int NT, int NL, int G, bool STORE,
-          int SIG>
+          int SIG, bool REV = false>
 __global__ void __launch_bounds__((W + 1 + NL) * 32, 1)
 plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     using L = LayoutT<T, A, K, X, W, SL, ST, NT>;
@@ -200,6 +204,11 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const long long ntiles = (long long)prm.ntiles;
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
+    static_assert(!REV || STORE, "the anticausal pass always stores");
+    // the tile the compute warps load element by element (REV: the first)
+    auto is_ragged = [&](long long j) -> bool { return last_ragged && j == (REV ? 0 : ntiles - 1); };
+    // first element of tile j in the arrays (REV: original tile ntiles-1-j)
+    auto tile_start = [&](long long j) -> long long { return (REV ? ntiles - 1 - j : j) * (long long)M; };
     // SIG != 0: the signature's tables are compile-time constants (plr_constsig.cuh)
     constexpr Tables<T, A> kTab = const_tables<T, A>(SIG, X, W, G);
     static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
@@ -249,9 +258,18 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     mbar_arrive(&full_L[s]);
                     break;
                 }
-                if (j == ntiles - 1 && last_ragged) { mbar_arrive(&full_L[s]); continue; }
+                if (is_ragged(j)) { mbar_arrive(&full_L[s]); continue; }
                 T* st = lstage + (size_t)s * SWL;
-                if (j == 0) {
+                if (REV) {                                      // the tile, its halo after it (zero beyond n)
+                    const long long o = tile_start(j);
+#pragma unroll
+                    for (int q = 0; q < kHalo; q++) {
+                        const unsigned long long i = (unsigned long long)(o + M + q);
+                        st[M + q] = (q < P && i < n) ? prm.x[i] : T(0);
+                    }
+                    mbar_arrive_tx(&full_L[s], M * sizeof(T));
+                    bulk_load(st, prm.x + (size_t)o, M * sizeof(T), &full_L[s], pol);
+                } else if (j == 0) {
 #pragma unroll
                     for (int q = 0; q < kHalo; q++)
                         st[q] = (q >= kHalo - P && prm.x_hist != nullptr) ? prm.x_hist[q - (kHalo - P)] : T(0);
@@ -272,8 +290,8 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 mbar_wait_poll(&full_T[sT], (uint32_t)((t / ST) & 1));
                 const long long jt = store_tile[sT];
                 if (jt >= ntiles) break;
-                if (STORE && !(jt == ntiles - 1 && last_ragged)) {
-                    bulk_store(prm.y + (size_t)jt * M, tstage + (size_t)sT * M, M * sizeof(T), pol);
+                if (STORE && !is_ragged(jt)) {
+                    bulk_store(prm.y + (size_t)tile_start(jt), tstage + (size_t)sT * M, M * sizeof(T), pol);
                     bulk_commit();
                     pend[np++] = sT;
                     if (np > ST - 1) {
@@ -399,12 +417,25 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (tid == 0) { slot_tile[slot] = j; *stop_pos = it; mbar_arrive(&agg_bar[slot]); }
             return j;
         }
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         const T* st = lstage + (size_t)s * SWL;
         const long long g0 = j * (long long)M + (long long)tid * X;
         // a1: my X elements (+ P halo)
         T xv[X + P];
-        if (!ragged) {
+        if (REV) {                                              // positions v: element o + M-1-v
+            const int v0 = tid * X - P;
+            if (!ragged) {
+#pragma unroll
+                for (int q = 0; q < X + P; q++) xv[q] = st[M - 1 - (v0 + q)];
+            } else {
+                const long long o = tile_start(j);
+#pragma unroll
+                for (int q = 0; q < X + P; q++) {
+                    const unsigned long long i = (unsigned long long)(o + M - 1 - (v0 + q));
+                    xv[q] = i < n ? prm.x[i] : T(0);
+                }
+            }
+        } else if (!ragged) {
             const T* base = st + kHalo + tid * X;
 #pragma unroll
             for (int q = 0; q < P; q++) xv[q] = base[q - P];
@@ -496,7 +527,7 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         // tile id read after the carry wait (tid 0 wrote it before agg_bar,
         // which the carry is ordered after; no barrier follows a stop)
         const long long j = slot_tile[slot];
-        const bool ragged = (j == ntiles - 1) && last_ragged;
+        const bool ragged = is_ragged(j);
         const long long g0 = j * (long long)M + (long long)tid * X;
         uint32_t w[CW];
         tmem_ld_n<CW>(tmem_w + (uint32_t)(slot * WQ * CW), w);
@@ -529,18 +560,18 @@ plr_scan_tmem_kernel(const __grid_constant__ ScanParams<T, A> prm) {
         mbar_wait(&empty_T[sT], (uint32_t)(((it / ST) & 1) ^ 1));   // store stage free
         if (!ragged) {
             if (STORE) {
-                T* base = tstage + (size_t)sT * M + tid * X;
+                T* stt = tstage + (size_t)sT * M;
 #pragma unroll
-                for (int u = 0; u < X; u++) base[u] = yv[u];
+                for (int u = 0; u < X; u++) stt[REV ? M - 1 - (tid * X + u) : tid * X + u] = yv[u];
             }
         } else if (STORE) {
 #pragma unroll
             for (int u = 0; u < X; u++) {
-                const long long i = g0 + u;
+                const long long i = REV ? tile_start(j) + M - 1 - (tid * X + u) : g0 + u;
                 if ((unsigned long long)i < n) prm.y[i] = yv[u];
             }
         }
-        if (prm.y_tail != nullptr) {
+        if (!REV && prm.y_tail != nullptr) {
             const long long lo = (long long)n - K;
             if (g0 + X > lo && g0 < (long long)n) {
 #pragma unroll

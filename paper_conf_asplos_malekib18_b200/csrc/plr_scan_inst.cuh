@@ -181,11 +181,21 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     if constexpr (kind == 2) {
         kern = &dev::plr_scan_rr_kernel<T, A, K, P, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS, PLR_RR_NL,
                                          C::U1 ? 1 : PLR_RR_G, STORE, SIG>;
+        if constexpr (STORE && SIG == 0) {               // the anticausal pass
+            if (la.reverse)
+                kern = &dev::plr_scan_rr_kernel<T, A, K, P, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS,
+                                                 PLR_RR_NL, C::U1 ? 1 : PLR_RR_G, STORE, 0, true>;
+        }
         smem = dev::LayoutR<T, A, K, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS>::bytes;
         threads = (PLR_RR_W + 1 + PLR_RR_NL) * 32;
     } else if constexpr (tmem) {
         using TC = TmCfg<T, A, K, C::U1>;
         kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, TC::G, STORE, SIG>;
+        if constexpr (STORE && SIG == 0) {               // the anticausal pass
+            if (la.reverse)
+                kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, TC::G,
+                                                   STORE, 0, true>;
+        }
         smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
         threads = (TC::W + 1 + TC::NL) * 32;
     } else {
@@ -197,12 +207,12 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
                 kern = &dev::plr_scan_kernel<T, A, K, P, C::X, C::W, C::S, C::D, C::NL, C::DEC, STORE, C::MINB, C::SEED,
                                              true>;
         }
-        if constexpr (C::DEC && STORE && C::DT) {         // forward DECAY pass with TMEM-parked map outputs
-            if (!la.reverse) {
-                kern = &dev::plr_scan_dect_kernel<T, A, K, P, C::X, C::W, PLR_DT_SL, PLR_DT_ST, PLR_DT_D, C::MINB>;
-                smem = dev::LayoutDT<T, A, K, C::X, C::W, PLR_DT_SL, PLR_DT_ST, PLR_DT_D + 1>::bytes;
-                threads = (C::W + 2) * 32;
-            }
+        if constexpr (C::DEC && STORE && C::DT) {         // DECAY passes with TMEM-parked map outputs
+            kern = la.reverse
+                ? &dev::plr_scan_dect_kernel<T, A, K, P, C::X, C::W, PLR_DT_SL, PLR_DT_ST, PLR_DT_D, C::MINB, true>
+                : &dev::plr_scan_dect_kernel<T, A, K, P, C::X, C::W, PLR_DT_SL, PLR_DT_ST, PLR_DT_D, C::MINB, false>;
+            smem = dev::LayoutDT<T, A, K, C::X, C::W, PLR_DT_SL, PLR_DT_ST, PLR_DT_D + 1>::bytes;
+            threads = (C::W + 2) * 32;
         }
     }
     // the > 48 KB dynamic shared memory opt-in is a per-device (context)

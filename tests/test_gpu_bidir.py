@@ -87,3 +87,20 @@ def test_reverse_full_size_decay(cuda_plr):
         worst = max(worst, float(np.max(np.abs(y - ref) / np.maximum(1, np.abs(ref)))))
     assert worst <= 1e-4, worst
     plan.close()
+
+
+@pytest.mark.parametrize("name", ["prefix", "tuple3", "order3", "lp3", "hp3"])
+def test_reverse_large_persistent(cuda_plr, name):
+    """The anticausal pass on the persistent kernels' REV instantiations (TMEM
+    k = 1, re-read k >= 2, TMEM-parked DECAY incl. fp64 accumulation) at
+    n = 2^27 - 3 (ragged first tile, thousands of tiles per launch), every
+    element against the oracle."""
+    import torch
+    sig = workloads.BY_NAME[name]
+    n = (1 << 27) - 3
+    x = workloads.host_input(n, sig.dtype, workloads.seed_for(18))
+    plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=n)
+    assert n > plan.info["small_max"]
+    y = plan.reverse(torch.from_numpy(x).cuda()).cpu().numpy()
+    check(y, oracle.anticausal(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s reverse n=%d" % (name, n))
+    plan.close()
