@@ -324,7 +324,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.lane_T = plan->d_lane;
     la.stats = plan->d_stats;
     la.grid = (int)grid;
-    la.sig = (plan->sig_kernel && !reverse) ? plan->pt.sig_id : 0;   // REV kernels read the parameter tables
+    la.sig = plan->sig_kernel ? plan->pt.sig_id : 0;
     la.store = store;
     la.unit1 = unit1;
     la.reverse = reverse;

@@ -181,20 +181,20 @@ cudaError_t launch_kps(const Tables<T, A>& tab, const LaunchArgs& la) {
     if constexpr (kind == 2) {
         kern = &dev::plr_scan_rr_kernel<T, A, K, P, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS, PLR_RR_NL,
                                          C::U1 ? 1 : PLR_RR_G, STORE, SIG>;
-        if constexpr (STORE && SIG == 0) {               // the anticausal pass
+        if constexpr (STORE) {                           // the anticausal pass
             if (la.reverse)
                 kern = &dev::plr_scan_rr_kernel<T, A, K, P, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS,
-                                                 PLR_RR_NL, C::U1 ? 1 : PLR_RR_G, STORE, 0, true>;
+                                                 PLR_RR_NL, C::U1 ? 1 : PLR_RR_G, STORE, SIG, true>;
         }
         smem = dev::LayoutR<T, A, K, PLR_RR_X, PLR_RR_W, PLR_RR_SA, PLR_RR_SB, PLR_RR_NS>::bytes;
         threads = (PLR_RR_W + 1 + PLR_RR_NL) * 32;
     } else if constexpr (tmem) {
         using TC = TmCfg<T, A, K, C::U1>;
         kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, TC::G, STORE, SIG>;
-        if constexpr (STORE && SIG == 0) {               // the anticausal pass
+        if constexpr (STORE) {                           // the anticausal pass
             if (la.reverse)
                 kern = &dev::plr_scan_tmem_kernel<T, A, K, P, TC::X, TC::W, TC::SL, TC::ST, TC::NT, TC::NL, TC::G,
-                                                   STORE, 0, true>;
+                                                   STORE, SIG, true>;
         }
         smem = dev::LayoutT<T, A, K, TC::X, TC::W, TC::SL, TC::ST, TC::NT>::bytes;
         threads = (TC::W + 1 + TC::NL) * 32;

@@ -195,3 +195,15 @@ def test_map_floor_reading_r20():
     lp3 = plr.Plan((0.008,), (2.4, -1.92, 0.512), "float32", n_max=0).info
     assert lp3["nyquist_gain"] == pytest.approx(0.008 / 5.832, rel=1e-5)
     assert plr.Plan((0.25, 0.5, 0.25), (0.8,), "float32", n_max=0).info["map_floor"] == float("inf")
+
+
+def test_plan_info_layout_host_only():
+    """plr_plan_info as the binding reads it (ctypes mirror of include/plr.h,
+    ABI 4): the fields after the doubles land where the C struct puts them.
+    A host-only plan reports the small-n cluster size (a compile-time
+    constant), no device state (0 clusters, 0 CTAs/SM, small_max 0)."""
+    info = plr.Plan((1,), (2, -1), "int32", n_max=0).info
+    assert info["small_cluster_ctas"] == 4
+    assert info["small_clusters"] == 0 and info["small_ctas_per_sm"] == 0 and info["small_max"] == 0
+    assert info["k"] == 2 and info["p"] == 0 and info["cls"] == "POLY"
+    assert info["nyquist_gain"] == 0.0 and info["map_floor"] == 0.0

@@ -6,6 +6,8 @@ mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/${TAG}_smi.txt
 timeout 1200 python -m pytest tests -m gpu -q --timeout 900 -p no:cacheprovider > gpurun_out/${TAG}_pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/${TAG}_pytest_gpu.log
 timeout 200 python tools/time_sigs.py $((1<<30)) > gpurun_out/${TAG}_times.log 2>&1
+timeout 300 python tools/time_sigs.py $((1<<30)) "" reverse > gpurun_out/${TAG}_times_reverse.log 2>&1
+timeout 300 python tools/time_sigs.py $((1<<30)) "" bidir > gpurun_out/${TAG}_times_bidir.log 2>&1
 timeout 900 python bench.py > gpurun_out/${TAG}_bench.log 2>&1; echo "bench rc=$?" >> gpurun_out/${TAG}_bench.log
 timeout 300 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/${TAG}_bench_ref.log 2>&1
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 3 --warmup 3 --no-extras > gpurun_out/${TAG}_bench_ncu.log 2>&1
