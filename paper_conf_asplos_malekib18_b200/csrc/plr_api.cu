@@ -328,6 +328,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.store = store;
     la.unit1 = unit1;
     la.reverse = reverse;
+    if (const char* lg = std::getenv("PLR_RR_LAG")) la.lag = std::atoi(lg);   // experiments
     la.stream = stream;
     cudaError_t e = launch_scan(plan->pt, la);
     if (e != cudaSuccess) {

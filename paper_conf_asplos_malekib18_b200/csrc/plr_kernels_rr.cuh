@@ -642,12 +642,17 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 
     // phase B of position nb reads its tile id from slot_tile[nb % NS]:
     // written at the end of phase A(nb), overwritten only by phase A(nb + NS)
+    // runtime lag Dr in [G-1, NS-1] (host: shorter at medium n, where the
+    // pipeline's fill and drain are a large share of the launch); phase B of
+    // a unit's first tile needs the unit's carries, i.e. phase A of its last
+    // tile, G-1 positions later
+    const int Dr = (prm.lag >= G - 1 && prm.lag < D) ? prm.lag : D;
     int na = 0, nb = 0;                                         // phases A / B done
-    for (; na < D; na++) {
+    for (; na < Dr; na++) {
         const long long ja = phaseA(na);
         if (ja >= ntiles) break;
     }
-    for (bool stop = na < D; !stop;) {
+    for (bool stop = na < Dr; !stop;) {
         const long long j = phaseA(na);
         phaseB(nb);
         nb++;

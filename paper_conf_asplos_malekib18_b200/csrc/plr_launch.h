@@ -28,6 +28,7 @@ struct LaunchArgs {
     bool unit1 = false;                 // look-back units of one tile (small n): the *_u1 kernels
     bool reverse = false;               // the anticausal recurrence (REV kernels: small-n, DECAY)
     bool cluster = false;               // small-n kernel: clusters of kSmallC tiles (cluster look-back)
+    int lag = 0;                        // re-read kernel: phase-B lag in tiles (0: NS-1)
     cudaStream_t stream;
     int* occupancy_out = nullptr;       // non-null: only report CTAs/SM of the kernel
 };
@@ -50,6 +51,7 @@ inline ScanParams<T, A> make_params(const Tables<T, A>& tab, const LaunchArgs& l
     prm.y_tail = static_cast<T*>(la.y_tail);
     prm.lane_T = static_cast<const A*>(la.lane_T);
     prm.stats = la.stats;
+    prm.lag = la.lag;
     prm.tab = tab;
     return prm;
 }
