@@ -52,6 +52,8 @@ struct plr_plan {
     size_t small_max = 0;               // n <= small_max: the small-n kernel (plr_kernels_small.cuh)
     int small_ctas = 0;                 // its CTAs per SM (all tiles resident: tile = blockIdx.x)
     int small_clusters = 0;             // co-resident clusters of kSmallC small-n CTAs (0: no cluster launches)
+    bool cluster_ok = true;             // PLR_SMALL_CLUSTER != 0 at plan creation
+    int rr_lag = 0;                     // PLR_RR_LAG at plan creation (0: the re-read kernel's NS-1)
     int reduce_ctas = 0;                // CTAs per SM of the reduce-only kernel (0: not available)
     unsigned long long* d_rd = nullptr; // its per-CTA records (kStatusMaxBytes each)
     void* d_scan_tmp = nullptr;         // CUB temp storage of the Scan comparator
@@ -281,9 +283,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
         if (resident_ok && la.ntiles <= (uint64_t)plan->num_sms * plan->small_ctas) la.dec_mask |= 0x100u;
         // non-decaying forward launches of several tiles whose clusters are
         // all co-resident: the cluster look-back (PLR_SMALL_CLUSTER=0 turns it off)
-        const char* ce = std::getenv("PLR_SMALL_CLUSTER");
-        const bool cluster_ok = ce == nullptr || ce[0] != '0';
-        if (cluster_ok && resident_ok && !reverse && !plan->pt.decay_s && la.ntiles >= 2 &&
+        if (plan->cluster_ok && resident_ok && !reverse && !plan->pt.decay_s && la.ntiles >= 2 &&
             (la.ntiles + kSmallC - 1) / kSmallC <= (uint64_t)plan->small_clusters) {
             la.cluster = true;
             la.dec_mask |= 0x100u;
@@ -328,7 +328,7 @@ static plr_status launch(plr_plan* plan, const void* x, void* y, size_t n, const
     la.store = store;
     la.unit1 = unit1;
     la.reverse = reverse;
-    if (const char* lg = std::getenv("PLR_RR_LAG")) la.lag = std::atoi(lg);   // experiments
+    la.lag = plan->rr_lag;
     la.stream = stream;
     cudaError_t e = launch_scan(plan->pt, la);
     if (e != cudaSuccess) {
@@ -467,6 +467,10 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
         }
     }
     plan->small_ctas = small_ctas;
+    // experiment switches, read once per plan: PLR_SMALL_CLUSTER=0 (no
+    // cluster launches), PLR_RR_LAG (the re-read kernel's phase-B lag)
+    if (const char* ce = std::getenv("PLR_SMALL_CLUSTER")) plan->cluster_ok = ce[0] != '0';
+    if (const char* lg = std::getenv("PLR_RR_LAG")) plan->rr_lag = std::atoi(lg);
     if (!plan->pt.decay_s && small_ctas >= 1) {
         if ((e = small_cluster_occupancy(plan->pt, &plan->small_clusters)) != cudaSuccess) {
             (void)cudaGetLastError();                          // no cluster launches on this device
@@ -475,7 +479,7 @@ plr_status plr_plan_create(plr_plan** out, const double* a, int p, const double*
                 std::fprintf(stderr, "plr: cluster occupancy query failed: %s\n", cudaGetErrorString(e));
         }
     }
-    plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default(plan->pt, plan->small_clusters)) : 0;
+    plan->small_max = small_ctas >= 1 ? std::min(n_max, small_max_default(plan->pt, plan->cluster_ok ? plan->small_clusters : 0)) : 0;
     const uint64_t m = (uint64_t)plan->pt.geo.tile(), ms = (uint64_t)plan->pt.geo_s.tile();
     plan->max_tiles = std::max<uint64_t>(1, (n_max + m - 1) / m);
     // Two status arrays: the persistent kernels' (their tiles up to n_max)
