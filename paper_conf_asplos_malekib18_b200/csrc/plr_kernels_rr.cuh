@@ -642,11 +642,13 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 
     // phase B of position nb reads its tile id from slot_tile[nb % NS]:
     // written at the end of phase A(nb), overwritten only by phase A(nb + NS)
-    // runtime lag Dr in [G-1, NS-1] (host: shorter at medium n, where the
-    // pipeline's fill and drain are a large share of the launch); phase B of
+    // runtime lag Dr in [max(1, G-1), NS-1] (prm.lag = 0: NS-1).  Phase B of
     // a unit's first tile needs the unit's carries, i.e. phase A of its last
-    // tile, G-1 positions later
-    const int Dr = (prm.lag >= G - 1 && prm.lag < D) ? prm.lag : D;
+    // tile, G-1 positions later; and the loop below runs phase B of position
+    // nb only after phase A of nb + Dr, so Dr >= 1 (with Dr = 0 the phase B
+    // of the stop position itself would wait for a carry that never comes)
+    constexpr int kMinLag = G - 1 > 1 ? G - 1 : 1;
+    const int Dr = (prm.lag >= kMinLag && prm.lag < D) ? prm.lag : D;
     int na = 0, nb = 0;                                         // phases A / B done
     for (; na < Dr; na++) {
         const long long ja = phaseA(na);

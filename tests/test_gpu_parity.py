@@ -476,3 +476,24 @@ def test_small_n_cluster_lookback(cuda_plr, name, cluster, monkeypatch):
     y2 = plan.continue_(torch.from_numpy(x[n1:].copy()).cuda(), x_hist=xh, y_hist=yh).cpu().numpy()
     check(np.concatenate([y1, y2]), ref, sig.dtype, "%s continuation cluster=%s" % (name, cluster))
     plan.close()
+
+
+@pytest.mark.parametrize("lag", ["0", "1", "5", "9"])
+def test_rr_runtime_lag(cuda_plr, lag, monkeypatch):
+    """The re-read kernel's phase-B lag at run time (PLR_RR_LAG, read at plan
+    creation; 0 = NS-1): the look-back units of one tile (medium n) and of
+    G tiles (large n), ragged, against the oracle.  A lag below max(1, G-1)
+    falls back to NS-1 (lag 0 once ran phase B of the stop position and hung)."""
+    import torch
+    monkeypatch.setenv("PLR_RR_LAG", lag)
+    for name in ("tuple2", "order3"):
+        sig = workloads.BY_NAME[name]
+        sizes = [(1 << 21) + 5, (1 << 23) + 77, (1 << 24) + 3]
+        x_all = workloads.host_input(max(sizes), sig.dtype, workloads.seed_for(19))
+        plan = cuda_plr.Plan(sig.a, sig.b, sig.dtype, n_max=max(sizes))
+        assert plan.info["small_max"] < sizes[0]
+        for n in sizes:
+            x = x_all[:n].copy()
+            y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+            check(y, oracle.recurrence(x, sig.a, sig.b, sig.dtype), sig.dtype, "%s n=%d lag=%s" % (name, n, lag))
+        plan.close()
