@@ -457,7 +457,10 @@ __device__ __forceinline__ void lookback_generic(const ScanParams<T, A>& prm, co
     long long c_wait = 0;
     // tiles per lane of a full window: 8 for small records, 4 when a record
     // has more than 2 words (keeps the window's registers in check)
-    constexpr int kT = StatusLayout<A, K, DEC>::NW <= 2 ? kTPL : kTPL / 2;
+#ifndef PLR_LB_WIDE_NW
+#define PLR_LB_WIDE_NW 2
+#endif
+    constexpr int kT = StatusLayout<A, K, DEC>::NW <= PLR_LB_WIDE_NW ? kTPL : kTPL / 2;
     constexpr int kLogT = kT == 8 ? 3 : 2;
     A acc[K];
     A Tacc[K * kMaxK];
