@@ -68,8 +68,8 @@ struct ScanParams {
     T* y_tail;                           // k slots y_{n-k}..y_{n-1} or null
     const A* lane_T;                     // [k*k][32]: T(X*l) per lane
     unsigned long long* stats;           // debug counters (PLR_STATS=1) or null
-    int lag;                             // re-read kernel: phase-B lag in tiles (0: its compile-time NS-1)
     Tables<T, A> tab;
+    int lag;                             // re-read kernel, PLR_RR_RUNTIME_LAG builds: phase-B lag in tiles (0: NS-1)
 };
 
 // Host-side planner result.

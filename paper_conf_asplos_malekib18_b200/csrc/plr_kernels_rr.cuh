@@ -72,6 +72,9 @@ struct RrCols { static constexpr int CW = K * AWords<A>::N; };
 // original tile ntiles-1-j read back to front, the ragged tile first (a
 // virtual full tile, zero beyond n), the map's halo after the tile (stage
 // layout [tile][halo]); phase B writes y into the stage in original order.
+// The REV paths are separate `if constexpr` branches, so the forward kernel's
+// code is the one measured before they existed (a shared formulation cost
+// tuple2 1.5 %, profiles/r04o_ab_rr.txt).
 template <typename T, typename A, int K, int P, int X, int W, int SA, int SB, int NS, int NL, int G, bool STORE,
           int SIG, bool REV = false>
 __global__ void __launch_bounds__((W + 1 + NL) * 32, 1)
@@ -125,10 +128,8 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     const unsigned long long n = prm.n;
     const bool last_ragged = (n % (unsigned long long)M) != 0;
     static_assert(!REV || STORE, "the anticausal pass always stores");
-    // the tile the compute warps load element by element (REV: the first)
-    auto is_ragged = [&](long long j) -> bool { return last_ragged && j == (REV ? 0 : ntiles - 1); };
-    // first element of tile j in the arrays (REV: original tile ntiles-1-j)
-    auto tile_start = [&](long long j) -> long long { return (REV ? ntiles - 1 - j : j) * (long long)M; };
+    // REV: first element of tile j in the arrays (original tile ntiles-1-j)
+    auto rev_start = [&](long long j) -> long long { return (ntiles - 1 - j) * (long long)M; };
     // SIG != 0: the signature's tables are compile-time constants (plr_constsig.cuh)
     constexpr Tables<T, A> kTab = const_tables<T, A>(SIG, X, W, G);
     static_assert(SIG == 0 || const_sig_k(SIG) == K, "signature order");
@@ -164,8 +165,8 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     };
     // TMA load of tile j (with its P-word halo) into stage st, completion on bar
     auto load_tile = [&](T* st, long long j, uint64_t* bar, uint64_t pol) {
-        if (REV) {                                              // the tile, its halo after it (zero beyond n)
-            const long long o = tile_start(j);
+        if constexpr (REV) {                                    // the tile, its halo after it (zero beyond n)
+            const long long o = rev_start(j);
 #pragma unroll
             for (int q = 0; q < kHalo; q++) {
                 const unsigned long long i = (unsigned long long)(o + M + q);
@@ -213,7 +214,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                     mbar_arrive(&fullA[s]);
                     break;
                 }
-                if (is_ragged(j)) { mbar_arrive(&fullA[s]); continue; }   // compute loads it
+                if (j == (REV ? 0 : ntiles - 1) && last_ragged) { mbar_arrive(&fullA[s]); continue; }   // compute loads it
                 load_tile(stA + (size_t)s * SWL, j, &fullA[s], pol);
             }
         } else if (lane == 1) {                                     // loader B (L2)
@@ -236,7 +237,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 const long long j = stop ? ntiles : slot_tile[slot];
                 if (j >= ntiles) break;
                 if (f >= SB) mbar_wait_poll(&emptyB[sb], (uint32_t)(((f / SB) - 1) & 1));
-                if (is_ragged(j)) { mbar_arrive(&fullB[sb]); continue; }
+                if (j == (REV ? 0 : ntiles - 1) && last_ragged) { mbar_arrive(&fullB[sb]); continue; }
                 if (!covers_tail(j)) { mbar_arrive(&fullB[sb]); continue; }   // reduce-only: phase B skipped
                 load_tile(stB + (size_t)sb * SWL, j, &fullB[sb], pol);
             }
@@ -267,9 +268,12 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
                 }
                 if (stop) { PLR_STAMP(13); break; }
                 const long long jt = store_tile[sb];
-                if (STORE && !is_ragged(jt))
-                    bulk_store(prm.y + (size_t)tile_start(jt), stB + (size_t)sb * SWL + (REV ? 0 : kHalo),
-                               M * sizeof(T), pol);
+                if constexpr (REV) {
+                    if (!(jt == 0 && last_ragged))
+                        bulk_store(prm.y + (size_t)rev_start(jt), stB + (size_t)sb * SWL, M * sizeof(T), pol);
+                } else if (STORE && !(jt == ntiles - 1 && last_ragged)) {
+                    bulk_store(prm.y + (size_t)jt * M, stB + (size_t)sb * SWL + kHalo, M * sizeof(T), pol);
+                }
                 bulk_commit();
                 bulk_wait_read<STQ - 1>();                          // stores up to t - STQ + 1 have read their stages
                 if (t - (STQ - 1) >= 0) mbar_arrive(&emptyB[(t - (STQ - 1)) % SB]);
@@ -387,20 +391,22 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
     // for the ragged last tile
     auto read_x = [&](const T* st, long long j, bool ragged, T (&xv)[X + P]) {
         const long long g0 = j * (long long)M + (long long)tid * X;
-        if (REV) {                                              // positions v: element o + M-1-v
+        if constexpr (REV) {                                    // positions v: element o + M-1-v
             const int v0 = tid * X - P;
             if (!ragged) {
 #pragma unroll
                 for (int q = 0; q < X + P; q++) xv[q] = st[M - 1 - (v0 + q)];
             } else {
-                const long long o = tile_start(j);
+                const long long o = rev_start(j);
 #pragma unroll
                 for (int q = 0; q < X + P; q++) {
                     const unsigned long long i = (unsigned long long)(o + M - 1 - (v0 + q));
                     xv[q] = i < n ? prm.x[i] : T(0);
                 }
             }
-        } else if (!ragged) {
+            return;
+        }
+        if (!ragged) {
             const T* base = st + kHalo + tid * X;
 #pragma unroll
             for (int q = 0; q < P; q++) xv[q] = base[q - P];
@@ -434,67 +440,27 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             if (tid == 0) { slot_tile[slot] = j; *stop_pos = it; mbar_arrive(&agg_bar[slot]); }
             return j;
         }
-        const bool ragged = is_ragged(j);
+        const bool ragged = (j == (REV ? 0 : ntiles - 1)) && last_ragged;
         T xv[X + P];
         read_x(stA + (size_t)s * SWL, j, ragged, xv);
         mbar_arrive(&emptyA[s]);                                // the stage may be refilled
         // a2: chunk end state with zero state (only the last K values matter)
-#ifndef PLR_RR_SPLIT
-#define PLR_RR_SPLIT 0
-#endif
-        A v[K];
-        if constexpr (PLR_RR_SPLIT && sizeof(A) == sizeof(T) && X >= 2 * K + 1) {
-            // two independent zero-state chains over [0, H) and [H, X) (twice
-            // the instruction-level parallelism of the serial chain), joined
-            // by the end state = h2 + T(X - H) h1, T(L)[q][r] = h^(r+1)_{L-1-q}
-            // = H[L-1-q][r] (Sec. 2.1)
-            constexpr int H = X / 2, H2 = X - H;
-            A h1[K], h2[K];
+        A hist[K];
 #pragma unroll
-            for (int r = 0; r < K; r++) { h1[r] = A(0); h2[r] = A(0); }
+        for (int r = 0; r < K; r++) hist[r] = A(0);
 #pragma unroll
-            for (int u = 0; u < H2; u++) {
-                if (u < H) {
-                    A acc = cvt<A, T>(fir(xv, u));
+        for (int u = 0; u < X; u++) {
+            A acc = cvt<A, T>(fir(xv, u));
 #pragma unroll
-                    for (int r = K; r >= 1; r--)
-                        if (u - r >= 0) acc = mad(tb.c[r - 1], h1[r - 1], acc);
+            for (int r = K; r >= 1; r--)
+                if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
 #pragma unroll
-                    for (int r = K - 1; r >= 1; r--) h1[r] = h1[r - 1];
-                    h1[0] = acc;
-                }
-                A acc2 = cvt<A, T>(fir(xv, H + u));
-#pragma unroll
-                for (int r = K; r >= 1; r--)
-                    if (u - r >= 0) acc2 = mad(tb.c[r - 1], h2[r - 1], acc2);
-#pragma unroll
-                for (int r = K - 1; r >= 1; r--) h2[r] = h2[r - 1];
-                h2[0] = acc2;
-            }
-#pragma unroll
-            for (int q = 0; q < K; q++) {
-                A acc = h2[q];
-#pragma unroll
-                for (int r = 0; r < K; r++) acc = mad(cvt<A, T>(tb.H[H2 - 1 - q][r]), h1[r], acc);
-                v[q] = acc;
-            }
-        } else {
-            A hist[K];
-#pragma unroll
-            for (int r = 0; r < K; r++) hist[r] = A(0);
-#pragma unroll
-            for (int u = 0; u < X; u++) {
-                A acc = cvt<A, T>(fir(xv, u));
-#pragma unroll
-                for (int r = K; r >= 1; r--)
-                    if (u - r >= 0) acc = mad(tb.c[r - 1], hist[r - 1], acc);
-#pragma unroll
-                for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
-                hist[0] = acc;
-            }
-#pragma unroll
-            for (int q = 0; q < K; q++) v[q] = hist[q];
+            for (int r = K - 1; r >= 1; r--) hist[r] = hist[r - 1];
+            hist[0] = acc;
         }
+        A v[K];
+#pragma unroll
+        for (int q = 0; q < K; q++) v[q] = hist[q];
         // a3: warp inclusive scan with T(X * 2^s)
 #pragma unroll
         for (int s2 = 0; s2 < 5; s2++) {
@@ -575,7 +541,7 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             mbar_arrive(&yfull[sb]);
             return;
         }
-        const bool ragged = is_ragged(j);
+        const bool ragged = (j == (REV ? 0 : ntiles - 1)) && last_ragged;
         const long long g0 = j * (long long)M + (long long)tid * X;
         uint32_t w[CW];
         tmem_ld_n<CW>(tmem_w + (uint32_t)(slot * WQ * CW), w);
@@ -613,15 +579,27 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
             yv[u] = cvt<T, A>(acc);
         }
         // a7: y into the stage (TMA store by the storer) or global (ragged)
-        if (!ragged) {
-            if (STORE) {
+        if constexpr (REV) {                                    // mirrored: the stage holds original order
+            if (!ragged) {
 #pragma unroll
-                for (int u = 0; u < X; u++) st[REV ? M - 1 - (tid * X + u) : kHalo + tid * X + u] = yv[u];
+                for (int u = 0; u < X; u++) st[M - 1 - (tid * X + u)] = yv[u];
+            } else {
+#pragma unroll
+                for (int u = 0; u < X; u++) {
+                    const long long i = rev_start(j) + M - 1 - (tid * X + u);
+                    if ((unsigned long long)i < n) prm.y[i] = yv[u];
+                }
+            }
+        } else if (!ragged) {
+            if (STORE) {
+                T* base = st + kHalo + tid * X;
+#pragma unroll
+                for (int u = 0; u < X; u++) base[u] = yv[u];
             }
         } else if (STORE) {
 #pragma unroll
             for (int u = 0; u < X; u++) {
-                const long long i = REV ? tile_start(j) + M - 1 - (tid * X + u) : g0 + u;
+                const long long i = g0 + u;
                 if ((unsigned long long)i < n) prm.y[i] = yv[u];
             }
         }
@@ -642,19 +620,25 @@ plr_scan_rr_kernel(const __grid_constant__ ScanParams<T, A> prm) {
 
     // phase B of position nb reads its tile id from slot_tile[nb % NS]:
     // written at the end of phase A(nb), overwritten only by phase A(nb + NS)
-    // runtime lag Dr in [max(1, G-1), NS-1] (prm.lag = 0: NS-1).  Phase B of
-    // a unit's first tile needs the unit's carries, i.e. phase A of its last
-    // tile, G-1 positions later; and the loop below runs phase B of position
-    // nb only after phase A of nb + Dr, so Dr >= 1 (with Dr = 0 the phase B
-    // of the stop position itself would wait for a carry that never comes)
+#ifndef PLR_RR_RUNTIME_LAG
+#define PLR_RR_RUNTIME_LAG 0        // experiment builds only: a runtime lag cost tuple2 0.7 % (r04m)
+#endif
+#if PLR_RR_RUNTIME_LAG
+    // runtime lag in [max(1, G-1), NS-1] (prm.lag = 0: NS-1): phase B of a
+    // unit's first tile needs phase A of its last tile, G-1 positions later,
+    // and phase B of position nb runs after phase A of nb + lag, so lag >= 1
+    // (lag 0 would run phase B of the stop position, which never gets a carry)
     constexpr int kMinLag = G - 1 > 1 ? G - 1 : 1;
-    const int Dr = (prm.lag >= kMinLag && prm.lag < D) ? prm.lag : D;
+    const int Dl = (prm.lag >= kMinLag && prm.lag < D) ? prm.lag : D;
+#else
+    constexpr int Dl = D;
+#endif
     int na = 0, nb = 0;                                         // phases A / B done
-    for (; na < Dr; na++) {
+    for (; na < Dl; na++) {
         const long long ja = phaseA(na);
         if (ja >= ntiles) break;
     }
-    for (bool stop = na < Dr; !stop;) {
+    for (bool stop = na < Dl; !stop;) {
         const long long j = phaseA(na);
         phaseB(nb);
         nb++;

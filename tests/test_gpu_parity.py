@@ -481,9 +481,10 @@ def test_small_n_cluster_lookback(cuda_plr, name, cluster, monkeypatch):
 @pytest.mark.parametrize("lag", ["0", "1", "5", "9"])
 def test_rr_runtime_lag(cuda_plr, lag, monkeypatch):
     """The re-read kernel's phase-B lag at run time (PLR_RR_LAG, read at plan
-    creation; 0 = NS-1): the look-back units of one tile (medium n) and of
-    G tiles (large n), ragged, against the oracle.  A lag below max(1, G-1)
-    falls back to NS-1 (lag 0 once ran phase B of the stop position and hung)."""
+    creation, honoured by PLR_RR_RUNTIME_LAG=1 builds; 0 = NS-1): the
+    look-back units of one tile (medium n) and of G tiles (large n), ragged,
+    against the oracle.  A lag below max(1, G-1) falls back to NS-1 (lag 0
+    once ran phase B of the stop position and hung)."""
     import torch
     monkeypatch.setenv("PLR_RR_LAG", lag)
     for name in ("tuple2", "order3"):
